@@ -1,0 +1,241 @@
+"""Pins of the D3Q19 LBM oracle (oracle/oracle.c) against facts the
+mathematics and physics fix: lattice identities (P6), equilibrium moments
+(P7), periodic conservation (P8), cavity mass conservation (P8b), uniform
+equilibrium / rest fixed points (P9), omega = 0 pure streaming (P10), an
+independently written pull-form brute force (P11) and shear-wave decay (P12).
+CPU only.
+"""
+from fractions import Fraction
+
+import numpy as np
+import pytest
+
+import stgen
+
+
+def _tables(oracle_lib):
+    e, wden, opp = oracle_lib.d3q19_tables()
+    w = [Fraction(1, int(d)) for d in wden]
+    return e, w, opp
+
+
+def test_lattice_identities(oracle_lib):
+    e, w, opp = _tables(oracle_lib)
+    assert sorted(map(tuple, e.tolist())) == sorted(
+        [(0, 0, 0)] + [v for v in __import__("itertools").product((-1, 0, 1), repeat=3)
+                       if 1 <= sum(map(abs, v)) <= 2])
+    assert sum(w) == 1
+    for a in range(3):
+        assert sum(w[i] * int(e[i, a]) for i in range(19)) == 0
+        for b in range(3):
+            s = sum(w[i] * int(e[i, a]) * int(e[i, b]) for i in range(19))
+            assert s == (Fraction(1, 3) if a == b else 0)
+            for c in range(3):
+                assert sum(w[i] * int(e[i, a]) * int(e[i, b]) * int(e[i, c]) for i in range(19)) == 0
+                for d in range(3):
+                    s4 = sum(w[i] * int(e[i, a] * e[i, b] * e[i, c] * e[i, d]) for i in range(19))
+                    dd = lambda p, q: 1 if p == q else 0
+                    assert s4 == Fraction(dd(a, b) * dd(c, d) + dd(a, c) * dd(b, d) + dd(a, d) * dd(b, c), 9)
+    for i in range(19):
+        assert opp[opp[i]] == i
+        assert (e[opp[i]] == -e[i]).all()
+    # DESIGN.md X10 ordering: opposite(i) = i+1 for odd i
+    assert all(opp[i] == i + 1 for i in range(1, 19, 2))
+    # crossing sets used by the Z-slab ghost logic
+    assert sorted(i for i in range(19) if e[i, 2] == 1) == [5, 11, 14, 15, 18]
+    assert sorted(i for i in range(19) if e[i, 2] == -1) == [6, 12, 13, 16, 17]
+
+
+@pytest.mark.parametrize("rho,u", [(1.0, (0.0, 0.0, 0.0)), (1.1, (0.05, -0.02, 0.03)), (0.9, (-0.1, 0.07, 0.0))])
+def test_equilibrium_moments(oracle_lib, rho, u):
+    e, _, _ = _tables(oracle_lib)
+    f = oracle_lib.feq(rho, *u, dtype=np.float64)
+    assert abs(f.sum() - rho) <= 4e-16 * 4
+    for a in range(3):
+        assert abs((f * e[:, a]).sum() - rho * u[a]) <= 4e-16 * 4
+        for b in range(3):
+            pab = (f * e[:, a] * e[:, b]).sum()
+            assert abs(pab - (rho / 3 * (a == b) + rho * u[a] * u[b])) <= 1e-15
+
+
+def _moments(f, e):
+    m = np.array([np.sum(f, dtype=np.float64)])
+    mom = [np.sum(f * e[:, a, None, None, None], dtype=np.float64) for a in range(3)]
+    return m[0], np.array(mom)
+
+
+@pytest.mark.parametrize("dtype,tol", [(np.float64, 1e-13), (np.float32, 3e-5)])
+def test_periodic_conservation(oracle_lib, dtype, tol):
+    e, _, _ = _tables(oracle_lib)
+    f0 = stgen.lbm_random(8, 8, 8, 3, dtype, amp=0.2)
+    flags = stgen.periodic_fluid_flags(8, 8, 8)
+    m0, p0 = _moments(f0.astype(np.float64), e)
+    f = oracle_lib.lbm(f0, flags, 1.3, 10, periodic=True)
+    m1, p1 = _moments(f.astype(np.float64), e)
+    assert abs(m1 - m0) <= tol * abs(m0)
+    assert np.max(np.abs(p1 - p0)) <= tol * abs(m0)
+    # the state did change (collision is active)
+    assert not np.allclose(f, f0)
+
+
+def test_uniform_equilibrium_fixed_point(oracle_lib):
+    rho0, u0 = 1.05, (0.04, -0.03, 0.02)
+    feq = oracle_lib.feq(rho0, *u0)
+    f0 = np.empty((19, 6, 5, 7))
+    f0[:] = feq[:, None, None, None]
+    f = oracle_lib.lbm(f0, stgen.periodic_fluid_flags(7, 5, 6), 1.6, 8, periodic=True)
+    assert np.max(np.abs(f - f0)) <= 1e-15
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_cavity_at_rest_exact_fixed_point(oracle_lib, dtype):
+    f0 = stgen.lbm_rest(9, 8, 7, dtype)
+    f = oracle_lib.lbm(f0, stgen.cavity_flags(9, 8, 7), 1.6, 6, u_lid=(0.0, 0.0, 0.0))
+    # fluid at rest with rho = 1: feq == f exactly except for rounding of w*rho*1
+    assert np.max(np.abs(f.astype(np.float64) - f0)) <= 2 * np.finfo(dtype).eps
+
+
+def test_omega0_is_pure_streaming(oracle_lib):
+    e, _, _ = _tables(oracle_lib)
+    f0 = stgen.lbm_random(7, 6, 5, 4, np.float64, amp=0.5)
+    T = 3
+    f = oracle_lib.lbm(f0, stgen.periodic_fluid_flags(7, 6, 5), 0.0, T, periodic=True)
+    for i in range(19):
+        ex, ey, ez = e[i]
+        ref = np.roll(f0[i], shift=(T * ez, T * ey, T * ex), axis=(0, 1, 2))
+        assert np.array_equal(f[i], ref), i
+
+
+def test_omega0_closed_box_round_trip(oracle_lib):
+    # in a closed box (walls only), omega = 0: a population leaving along +x
+    # bounces back and the whole state returns after a period of 2*(n_fluid)
+    nx, ny, nz = 6, 5, 5
+    flags = stgen.cavity_flags(nx, ny, nz)
+    flags[flags == stgen.LID] = stgen.WALL
+    f0 = stgen.lbm_random(nx, ny, nz, 5, np.float64, amp=0.5)
+    # fluid extent 4 x 3 x 3: periods 8 (x), 6 (y, z); lcm over diagonals = 24
+    f = oracle_lib.lbm(f0, flags, 0.0, 24)
+    assert np.array_equal(f, f0)
+    f_half = oracle_lib.lbm(f0, flags, 0.0, 4)
+    assert not np.array_equal(f_half, f0)
+
+
+@pytest.mark.parametrize("dtype,tol", [(np.float64, 1e-13), (np.float32, 2e-5)])
+def test_cavity_mass_conservation(oracle_lib, dtype, tol):
+    nx, ny, nz = 9, 8, 7
+    flags = stgen.cavity_flags(nx, ny, nz)
+    f0 = stgen.lbm_random(nx, ny, nz, 6, dtype)
+    fl = flags == stgen.FLUID
+    m0 = np.sum(f0.astype(np.float64)[:, fl])
+    f = oracle_lib.lbm(f0, flags, 1.6, 6, u_lid=(0.05, 0.0, 0.0))
+    m1 = np.sum(f.astype(np.float64)[:, fl])
+    assert abs(m1 - m0) <= tol * m0
+    # lid drives +x: from rest, the mean x-velocity becomes positive
+    e, _, _ = _tables(oracle_lib)
+    fr = oracle_lib.lbm(stgen.lbm_rest(nx, ny, nz, np.float64), flags, 1.6, 6, u_lid=(0.05, 0, 0))
+    jx = np.sum((fr * e[:, 0, None, None, None])[:, fl])
+    assert jx > 0
+    # walls only (no lid) from rest: nothing moves
+    assert np.max(np.abs(oracle_lib.lbm(stgen.lbm_rest(nx, ny, nz, np.float64), flags, 1.6, 6,
+                                        u_lid=(0, 0, 0)) - stgen.lbm_rest(nx, ny, nz, np.float64))) < 1e-15
+
+
+def _collide_np(f, omega, dtype):
+    """vectorised BGK in the operation order of DESIGN.md X20 (for P11)."""
+    T = np.dtype(dtype).type
+    E = [(0, 0, 0), (1, 0, 0), (-1, 0, 0), (0, 1, 0), (0, -1, 0), (0, 0, 1), (0, 0, -1),
+         (1, 1, 0), (-1, -1, 0), (1, -1, 0), (-1, 1, 0), (1, 0, 1), (-1, 0, -1), (1, 0, -1),
+         (-1, 0, 1), (0, 1, 1), (0, -1, -1), (0, 1, -1), (0, -1, 1)]
+    W = [3] + [18] * 6 + [36] * 12
+    rho = f[0].copy()
+    for i in range(1, 19):
+        rho = rho + f[i]
+    j = []
+    for a in range(3):
+        acc = None
+        for i in range(19):
+            if E[i][a] == 0:
+                continue
+            term = f[i] if E[i][a] > 0 else -f[i]
+            acc = term.copy() if acc is None else acc + term
+        j.append(acc)
+    u = [ja / rho for ja in j]
+    usq = (u[0] * u[0] + u[1] * u[1]) + u[2] * u[2]
+    usq15 = T(1.5) * usq
+    out = np.empty_like(f)
+    for i in range(19):
+        eu = None
+        for a in range(3):
+            if E[i][a]:
+                v = u[a] if E[i][a] > 0 else -u[a]
+                eu = v if eu is None else eu + v
+        if eu is None:
+            eu = np.zeros_like(rho)
+        w = T(1) / T(W[i])
+        feq = (w * rho) * (((T(1) + T(3) * eu) + (T(4.5) * eu) * eu) - usq15)
+        out[i] = f[i] - T(omega) * (f[i] - feq)
+    return out, E, W
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_pull_form_bruteforce(oracle_lib, dtype):
+    """P11: f_new_i(y) = C(f)_i(y - e_i) if that cell is FLUID, else the
+    bounce-back f*_opp(i)(y) (+ 6 w_i e_i.u_lid for a LID source); non-fluid
+    cells copy.  Written as a gather, independently of the push loop."""
+    T = np.dtype(dtype).type
+    nx, ny, nz = 8, 8, 8
+    flags = stgen.cavity_flags(nx, ny, nz)
+    f = stgen.lbm_random(nx, ny, nz, 12, dtype)
+    omega, ulid = 1.6, (0.05, 0.0, 0.0)
+    ref = f.copy()
+    for step in range(2):
+        fs, E, W = _collide_np(ref, omega, dtype)
+        new = ref.copy()
+        for z in range(nz):
+            for y in range(ny):
+                for x in range(nx):
+                    if flags[z, y, x] != stgen.FLUID:
+                        continue
+                    for i in range(19):
+                        ex, ey, ez = E[i]
+                        sx, sy, sz = x - ex, y - ey, z - ez
+                        src = flags[sz, sy, sx]
+                        if src == stgen.FLUID:
+                            new[i, z, y, x] = fs[i, sz, sy, sx]
+                        else:
+                            o = i + 1 if i % 2 == 1 else i - 1
+                            v = fs[o, z, y, x]
+                            if src == stgen.LID:
+                                # push rule: f*_o - (6 w_o)(e_o . u_lid); e_o = -e_i
+                                eo = E[o]
+                                eu = None
+                                for a in range(3):
+                                    if eo[a]:
+                                        t = T(ulid[a]) if eo[a] > 0 else -T(ulid[a])
+                                        eu = t if eu is None else eu + t
+                                v = v - (T(6) * (T(1) / T(W[o]))) * eu
+                            new[i, z, y, x] = v
+        ref = new
+    got = oracle_lib.lbm(f, flags, omega, 2, u_lid=ulid)
+    assert np.array_equal(got, ref)
+
+
+def test_shear_wave_decay(oracle_lib):
+    """P12: u_x = U sin(2 pi z / nz) decays as exp(-nu k^2 t), nu = (1/omega - 1/2)/3."""
+    nz, U, omega, T = 64, 0.01, 1.0, 300
+    e, _, _ = _tables(oracle_lib)
+    z = np.arange(nz)
+    ux = U * np.sin(2 * np.pi * z / nz)
+    f0 = np.empty((19, nz, 1, 1))
+    for k in range(nz):
+        f0[:, k, 0, 0] = oracle_lib.feq(1.0, ux[k], 0.0, 0.0)
+    f = oracle_lib.lbm(f0, stgen.periodic_fluid_flags(1, 1, nz), omega, T, periodic=True)
+    rho = f.sum(0)[:, 0, 0]
+    uxt = (f * e[:, 0, None, None, None]).sum(0)[:, 0, 0] / rho
+    amp = 2 * np.mean(uxt * np.sin(2 * np.pi * z / nz))
+    nu = (1 / omega - 0.5) / 3
+    expect = U * np.exp(-nu * (2 * np.pi / nz) ** 2 * T)
+    assert abs(amp / expect - 1) < 0.01
+    # wrong viscosity (e.g. a dropped 1/2) would be far off
+    wrong = U * np.exp(-(1 / omega) / 3 * (2 * np.pi / nz) ** 2 * T)
+    assert abs(amp / wrong - 1) > 0.05
