@@ -1,0 +1,372 @@
+#!/usr/bin/env python
+"""bench.py — throughput of the 3.5D-blocked sweeps on B200 (BASELINE.json metric).
+
+Headline (N=1): BASELINE configs[1], 7-point stencil FP32 256^3, T=100, with
+dim_T chosen by measurement (one pass of every dim_T in 1..8, the fastest is
+timed).  One step = one st7_run call (T=100 Jacobi steps, all §8(a) rows of
+the 7-point path: planner, prolog, TMA plane loads, on-chip levels, final
+store, sweep driver).  value = interior updates per second over all ranks
+(Mupdates/s; X3: an update is one interior point advanced one time step).
+
+Extra lines inside the same JSON object: FP64 256^3, FP32 512^3 (configs[3]
+per-GPU size) and the D3Q19 cavity 256^3 (configs[2], MLUPS).
+
+Timing: W warm-up steps, then K steps each bracketed by CUDA events on the
+plan's stream; L2 (126 MB) is flushed by writing a 512 MiB buffer between
+timed steps (outside the timed region); max over ranks.  e2e repeats the
+headline through the C ABI with HOST (pinned) buffers, copies inside the
+timed region.  `--impl reference` times the CPU oracle on the host cores.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
+TRAFFIC_PATH = os.path.join(ROOT, "profiles", "traffic.json")
+SM_COUNT = 148
+FP32_LANES, FP64_LANES = 128, 64
+ST7_OPS = 7            # FP instructions per 7-point update: 5 add, 1 mul, 1 fma (8 flops)
+LBM_BYTES = {4: 153, 8: 305}   # (19*2*E + 1) per LBM update at dim_T = 1 (X12)
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--n", type=int, default=256)
+    ap.add_argument("--T", type=int, default=100)
+    ap.add_argument("--dim-t", type=int, default=0, help="0 = choose by measurement")
+    ap.add_argument("--no-extras", action="store_true")
+    return ap.parse_args()
+
+
+def peaks():
+    try:
+        with open(PEAKS_PATH) as fh:
+            d = json.load(fh)
+        return float(d["hbm_gbs"]), float(d.get("sm_max_mhz", 1965.0)), "measured"
+    except Exception:
+        return 6650.0, 1965.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi style clock / throttle sampling during the timed region (pynvml)."""
+
+    def __init__(self, dev: int):
+        self.dev = dev
+        self.samples = []
+        self.reasons = set()
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self._t = None
+
+    def __enter__(self):
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            h = pynvml.nvmlDeviceGetHandleByIndex(self.dev)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+            names = {
+                "hw_slowdown": getattr(pynvml, "nvmlClocksThrottleReasonHwSlowdown", 0x8),
+                "hw_thermal_slowdown": getattr(pynvml, "nvmlClocksThrottleReasonHwThermalSlowdown", 0x40),
+                "sw_thermal_slowdown": getattr(pynvml, "nvmlClocksThrottleReasonSwThermalSlowdown", 0x20),
+                "sw_power_cap": getattr(pynvml, "nvmlClocksThrottleReasonSwPowerCap", 0x4),
+            }
+
+            def run():
+                while not self._stop.is_set():
+                    try:
+                        self.samples.append(pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM))
+                        r = pynvml.nvmlDeviceGetCurrentClocksThrottleReasons(h)
+                        for k, bit in names.items():
+                            if r & bit:
+                                self.reasons.add(k)
+                    except Exception:
+                        pass
+                    time.sleep(0.05)
+
+            self._t = threading.Thread(target=run, daemon=True)
+            self._t.start()
+        except Exception:
+            self._t = None
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def summary(self):
+        s = sorted(self.samples)
+        return {"sm_mhz": s[len(s) // 2] if s else None, "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(s)}
+
+
+def load_traffic(key):
+    try:
+        with open(TRAFFIC_PATH) as fh:
+            return json.load(fh).get(key)
+    except Exception:
+        return None
+
+
+# ----------------------------------------------------------------------------
+# reference arm: the CPU oracle as it stands, on the host cores
+# ----------------------------------------------------------------------------
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    import oracle
+    import stgen
+    n = args.n
+    a = stgen.grid7(n, n, n, 2, np.float32)
+    Ts = 2  # bounded sample per step: 2 sweeps of the 256^3 grid
+    for _ in range(max(1, args.warmup)):
+        oracle.st7(a, 0.4, 0.1, 1)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.st7(a, 0.4, 0.1, Ts)
+    dt = time.perf_counter() - t0
+    upd = (n - 2) ** 3 * Ts * args.steps
+    v = upd / dt / 1e6
+    cores = oracle.num_threads()
+    line = {
+        "impl": "reference", "metric": "Mupdates/s (7-pt)", "value": round(v, 2), "unit": "Mupdates/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(dt / args.steps * 1e3, 3), "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f32", "data": "synthetic (splitmix64 U[0,1), seed 2)",
+        "config": {"workload": f"7-point FP32 {n}^3 (configs[1]); each step a bounded sample of T={Ts} sweeps",
+                   "grid": [n, n, n], "T_sample": Ts},
+        "cpu_baseline": {"value": round(v, 2), "unit": "Mupdates/s", "cores": cores, "kind": "oracle",
+                         "sample": f"{n}^3 FP32, {Ts} Jacobi sweeps per step, {args.steps} steps"},
+        "e2e": {"value": round(v, 2), "unit": "Mupdates/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline_7pt(n):
+    """the oracle timed on a bounded sample (~10 s) of the headline workload."""
+    import oracle
+    import stgen
+    a = stgen.grid7(n, n, n, 2, np.float32)
+    t0 = time.perf_counter()
+    oracle.st7(a, 0.4, 0.1, 1)
+    t1 = time.perf_counter() - t0
+    Ts = int(max(1, min(100, round(10.0 / max(t1, 1e-3)))))
+    t0 = time.perf_counter()
+    oracle.st7(a, 0.4, 0.1, Ts)
+    dt = time.perf_counter() - t0
+    return {"value": round((n - 2) ** 3 * Ts / dt / 1e6, 2), "unit": "Mupdates/s",
+            "cores": oracle.num_threads(), "kind": "oracle",
+            "sample": f"7-point FP32 {n}^3, T={Ts} sweeps ({dt:.1f} s), OpenMP over z"}
+
+
+# ----------------------------------------------------------------------------
+# our arm
+# ----------------------------------------------------------------------------
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+    import stgen
+    import paper_conf_sc_nguyensckd10_b200 as st
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def max_over_ranks(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    hbm_gbs, sm_max, peak_src = peaks()
+    stream = torch.cuda.Stream()
+    flush = torch.empty(512 * 2 ** 20 // 4, dtype=torch.float32, device="cuda")
+
+    def l2_flush():
+        flush.fill_(1.0)
+
+    def time_steps(run, steps, warmup):
+        """returns (total device ms, per-step ms list); events on `stream`."""
+        for _ in range(warmup):
+            run()
+        torch.cuda.synchronize()
+        tot = 0.0
+        per = []
+        for _ in range(steps):
+            l2_flush()
+            torch.cuda.synchronize()
+            barrier()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            run()
+            e1.record(stream)
+            e1.synchronize()
+            ms = e0.elapsed_time(e1)
+            per.append(ms)
+            tot += ms
+        torch.cuda.synchronize()
+        return tot, per
+
+    # ------------------------------------------------------------------ 7-point
+    def st7_case(n, T, dtype, dim_t_fixed=0, steps=args.steps, warmup=args.warmup, choose=range(1, 9)):
+        tdt = torch.float32 if dtype == np.float32 else torch.float64
+        a0 = torch.from_numpy(stgen.grid7(n, n, n, 2 + rank, dtype)).cuda()
+        x = a0.clone()
+        y = torch.empty_like(a0)
+        sweep = {}
+        if dim_t_fixed:
+            best = dim_t_fixed
+        else:
+            for d in choose:
+                with st.Plan(n, n, n, tdt, d) as p:
+                    p.set_stream(stream)
+                    p.st7(x, y, 0.4, 0.1, T)
+                    torch.cuda.synchronize()
+                    tms, _ = time_steps(lambda: p.st7(x, y, 0.4, 0.1, T), 2, 0)
+                    sweep[d] = round((n - 2) ** 3 * T / (tms / 2 / 1e3) / 1e6, 1)
+            best = max(sweep, key=sweep.get)
+        p = st.Plan(n, n, n, tdt, best)
+        p.set_stream(stream)
+        tms, per = time_steps(lambda: p.st7(x, y, 0.4, 0.1, T), steps, warmup)
+        launches = p.last_launches()
+        info = p.info()
+        ms = max_over_ranks(tms / steps)
+        upd = (n - 2) ** 3 * T
+        return p, best, sweep, ms, upd, launches, info, (a0, x, y)
+
+    with ClockSampler(local) as clk:
+        n, T = args.n, args.T
+        p7, D, sweep, ms, upd, launches, info, bufs = st7_case(n, T, np.float32, args.dim_t)
+        value = upd * world / (ms / 1e3) / 1e6
+        per_launch_ms = ms / launches
+        d_eff = info["dim_t_sweep"]
+        # roofline of the dominant kernel (st7_35d): both roofs, report the binding one
+        ops_peak = SM_COUNT * FP32_LANES * sm_max * 1e6 / 1e12          # T FP32 lane-ops/s
+        achieved_ops = ST7_OPS * upd / (ms / 1e3) / 1e12
+        bytes_per_upd = 8.0 / D
+        achieved_gbs = bytes_per_upd * upd / (ms / 1e3) / 1e9
+        hbm_roof_upd = hbm_gbs * 1e9 / bytes_per_upd
+        alu_roof_upd = ops_peak * 1e12 / ST7_OPS
+        traffic = load_traffic(f"st7_f32_{n}_D{D}")
+        r_alu = {"bound": "alu", "achieved": round(achieved_ops, 3), "peak": round(ops_peak, 2),
+                 "unit": "Top/s (FP32 lane-instructions; 7 per update)",
+                 "frac": round(achieved_ops / ops_peak, 4), "traffic": traffic,
+                 "peak_source": f"148 SM x 128 FP32 lanes x {sm_max:.0f} MHz (clocks.max.sm)"}
+        r_hbm = {"bound": "hbm", "achieved": round(achieved_gbs, 1), "peak": hbm_gbs, "unit": "GB/s",
+                 "frac": round(achieved_gbs / hbm_gbs, 4), "traffic": traffic,
+                 "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_src}); algorithmic 8/dim_T B/update"}
+        roof, alt = (r_hbm, r_alu) if hbm_roof_upd < alu_roof_upd else (r_alu, r_hbm)
+
+    # ------------------------------------------------------------------ e2e (host buffers)
+    a_host = torch.from_numpy(stgen.grid7(n, n, n, 2 + rank, np.float32)).pin_memory()
+    o_host = torch.empty_like(a_host).pin_memory()
+    hin, hout = a_host.numpy(), o_host.numpy()
+    for _ in range(max(1, args.warmup)):
+        st.st7_run(p7.h, hin, hout, 0.4, 0.1, T)
+    e2e_t = 0.0
+    for _ in range(args.steps):
+        barrier()
+        t0 = time.perf_counter()
+        st.st7_run(p7.h, hin, hout, 0.4, 0.1, T)
+        e2e_t += time.perf_counter() - t0
+    e2e_ms = max_over_ranks(e2e_t / args.steps * 1e3)
+    grid_bytes = n ** 3 * 4
+
+    extras = {}
+    if not args.no_extras:
+        # FP64 256^3 (configs[1] FP64)
+        _, D64, sw64, ms64, upd64, l64, inf64, _ = st7_case(n, T, np.float64, 0, steps=3, warmup=1,
+                                                           choose=range(1, 9))
+        extras["st7_f64_256"] = {"value": round(upd64 * world / (ms64 / 1e3) / 1e6, 1), "unit": "Mupdates/s",
+                                 "dim_T": D64, "dim_T_sweep": sw64, "ms_per_step": round(ms64, 3),
+                                 "frac_alu": round(ST7_OPS * upd64 / (ms64 / 1e3) /
+                                                   (SM_COUNT * FP64_LANES * sm_max * 1e6), 4)}
+        # FP32 512^3 (configs[3] per-GPU size)
+        _, D5, sw5, ms5, upd5, l5, inf5, _ = st7_case(512, T, np.float32, 0, steps=3, warmup=1,
+                                                      choose=range(1, 9))
+        extras["st7_f32_512"] = {"value": round(upd5 * world / (ms5 / 1e3) / 1e6, 1), "unit": "Mupdates/s",
+                                 "dim_T": D5, "dim_T_sweep": sw5, "ms_per_step": round(ms5, 3),
+                                 "frac_alu": round(ST7_OPS * upd5 / (ms5 / 1e3) / (ops_peak * 1e12), 4),
+                                 "info": inf5}
+        # LBM D3Q19 cavity 256^3 (configs[2])
+        for dtn, dt_np, tdt in (("f32", np.float32, torch.float32), ("f64", np.float64, torch.float64)):
+            nl, Tl = 256, 100
+            flags = torch.from_numpy(stgen.cavity_flags(nl, nl, nl)).cuda()
+            f0 = torch.from_numpy(stgen.lbm_rest(nl, nl, nl, dt_np)).cuda()
+            fa, fb = f0.clone(), torch.empty_like(f0)
+            with st.Plan(nl, nl, nl, tdt, 1) as pl:
+                pl.set_stream(stream)
+                pl.set_lid(0.05, 0.0, 0.0)
+                tl, _ = time_steps(lambda: pl.lbm(fa, fb, 1.6, Tl, flags), 2, 1)
+                msl = max_over_ranks(tl / 2)
+                cells = (nl - 2) ** 3
+                mlups = cells * Tl * world / (msl / 1e3) / 1e6
+                E = 4 if dtn == "f32" else 8
+                gbs = LBM_BYTES[E] * cells * Tl / (msl / 1e3) / 1e9
+                extras[f"lbm_{dtn}_256"] = {"value": round(mlups, 1), "unit": "MLUPS", "dim_T": 1,
+                                            "ms_per_step": round(msl, 3),
+                                            "roofline": {"bound": "hbm", "achieved": round(gbs, 1),
+                                                         "peak": hbm_gbs, "unit": "GB/s",
+                                                         "frac": round(gbs / hbm_gbs, 4)},
+                                            "launches": pl.last_launches()}
+            del fa, fb, f0, flags
+    cpu = cpu_baseline_7pt(n) if (rank == 0 and world >= 1) else None
+
+    if rank == 0:
+        line = {
+            "metric": "Mupdates/s (7-pt)", "value": round(value, 1), "unit": "Mupdates/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(ms, 4), "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic (splitmix64 U[0,1) grid, seed 2; alpha=0.4 beta=0.1)",
+            "config": {"workload": f"7-point stencil FP32 {n}^3, T={T} (BASELINE configs[1]); "
+                                   f"dim_T chosen by measurement",
+                       "grid": [n, n, n], "T": T, "dim_T": D, "dim_T_sweep_Mupd": sweep,
+                       "parallelism": f"replicas x{world}" if world > 1 else "single",
+                       "l2": "flushed between timed steps (512 MiB write)",
+                       "plan": info},
+            "roofline": roof, "roofline_alt": alt,
+            "e2e": {"value": round(upd * world / (e2e_ms / 1e3) / 1e6, 1), "unit": "Mupdates/s",
+                    "h2d_bytes_per_step": grid_bytes, "d2h_bytes_per_step": grid_bytes,
+                    "ms_per_step": round(e2e_ms, 3)},
+            "gpu_launches": launches * args.steps,
+            "kernel_ms_per_launch": round(per_launch_ms, 5),
+            "clocks": clk.summary(),
+            "cpu_baseline": cpu,
+            "extras": extras,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,189 @@
+/*
+ * st35d.h — C ABI of the B200 (sm_100a) 3.5D-blocked stencil sweeps.
+ *
+ * The operations are the two kernels of Nguyen et al., "3.5-D Blocking
+ * Optimization for Stencil Computations on Modern CPUs and GPUs" (SC'10),
+ * /root/reference/PAPER.md (cited P:<line>):
+ *   - 7-point Jacobi stencil (§IV-A1, equation at; Jacobi two-grid
+ *     sweep P:95; fixed boundary P:195),
+ *   - D3Q19 lattice-Boltzmann collide+stream (§IV-B, steps 1-4 at P:125-132),
+ * both executed by the 3.5D-blocked sweep of §V (2.5D spatial blocking of an
+ * XY tile streamed along Z, plus dim_T time steps kept on chip,
+ * P:183-255).  Blocking only reorders the computation, so the result
+ * is that of T plain Jacobi sweeps.
+ *
+ * Memory layout: X fastest, then Y, then Z:
+ *     idx(x,y,z) = (z*ny + y)*nx + x
+ * LBM populations are SoA: f[i][z][y][x], i = 0..18, in the
+ * velocity order of DESIGN.md (0 rest; 1..6 = +x,-x,+y,-y,+z,-z; 7..18 the
+ * edge directions; opposite(i) = i+1 for odd i).  flags[z][y][x] is uint8:
+ * 0 FLUID, 1 WALL (half-way bounce-back), 2 LID (moving wall, Ladd, rho_w=1).
+ *
+ * Ownership: the library never owns the grid buffers.  Pointers may be
+ * DEVICE memory (the fast path: the call only enqueues kernels on the plan's
+ * stream and returns) or HOST memory (pageable or pinned: the call copies to
+ * plan-owned device scratch, runs, copies the result back and synchronises
+ * before returning).  Host and device pointers may not be mixed in one call.
+ *
+ * Errors: every argument is checked before anything is launched; on error
+ * nothing is written, the call returns a negative ST_E* code and
+ * st_last_error() returns a thread-local message.  Device-side faults of an
+ * asynchronous (device-pointer) run surface at the next call or at
+ * st_plan_sync().  A plan is not thread-safe.
+ */
+#ifndef ST35D_H
+#define ST35D_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct st_plan st_plan; /* opaque: owns streams, events, scratch, comm */
+
+typedef enum { ST_F32 = 0, ST_F64 = 1 } st_dtype;
+
+enum {
+    ST_OK = 0,
+    ST_EINVAL = -1,       /* bad argument (sizes, dim_T, T, omega, NULL pointer, aliasing) */
+    ST_ENOMEM = -2,       /* device or host allocation failed                           */
+    ST_ECUDA = -3,        /* CUDA runtime / driver error (incl. deferred device faults) */
+    ST_ENCCL = -4,        /* NCCL error in the Z-slab ghost exchange                    */
+    ST_EUNSUPPORTED = -5  /* valid request this build does not handle (see message)     */
+};
+
+enum { ST_FLUID = 0, ST_WALL = 1, ST_LID = 2 };
+
+/* Maximum temporal blocking depth compiled into this build. */
+#define ST_MAX_DIM_T 8
+
+/*
+ * st_plan_create — plan a sweep over an nx*ny*nz grid of `dtype` with
+ * temporal blocking depth dim_T (number of time steps kept on chip per
+ * sweep; eq. (3) P:225 says dim_T >= eta = ceil(gamma/Gamma)).
+ * Requirements: nx, ny, nz >= 3; 1 <= dim_T <= ST_MAX_DIM_T;
+ * nx*sizeof(dtype) a multiple of 16 bytes (TMA row-pitch rule).
+ * The planner chooses the XY tile (eq. (1)/(4) analog for the on-chip bytes
+ * of one SM) and the persistent grid that gives every CTA the same number of
+ * tile-planes (flexible load balance).
+ * nz is the GLOBAL number of planes even in distributed mode.
+ * Returns NULL on error (st_last_error() says why).  Needs a CUDA device.
+ */
+st_plan* st_plan_create(int nx, int ny, int nz, st_dtype dtype, int dim_T);
+
+/*
+ * st7_run — out = A(T): T Jacobi sweeps of the 7-point stencil
+ *     B = alpha*A + beta*(A[x-1]+A[x+1]+A[y-1]+A[y+1]+A[z-1]+A[z+1])
+ * applied to every interior point; the shell x in {0,nx-1}, y in {0,ny-1},
+ * z in {0,nz-1} is Dirichlet-fixed and copied.  alpha, beta are
+ * rounded once to the plan dtype.  `in` and `out` are nx*ny*nz elements of
+ * the plan dtype, must not overlap, and 16-byte aligned (device).  `in` is
+ * SCRATCH: it is overwritten when more than one sweep runs (the two grids
+ * ping-pong; no third grid is allocated).  T = 0 copies in to out.
+ * In distributed mode (st_plan_set_dist) each rank passes its own slab
+ * buffers of (nz_local + 2*g) planes, g = st_plan_ghost_planes(plan).
+ */
+int st7_run(st_plan* plan, const void* in, void* out, double alpha, double beta, int T);
+
+/*
+ * lbm_d3q19_run — f_dst = state after T D3Q19 steps of f_src,
+ * BGK single-relaxation collision with relaxation rate omega (0 <= omega < 2;
+ * omega = 0 is pure streaming), push semantics: the stored state is
+ * post-stream, pre-collision.  FLUID cells collide and propagate; a link into
+ * a WALL cell bounces back (half-way); a link into a LID cell bounces back
+ * with the Ladd correction -6*w_i*(e_i . u_lid) (rho_w = 1); non-FLUID cells
+ * keep their 19 values.  f_src / f_dst are 19*nx*ny*nz elements (SoA), flags
+ * nx*ny*nz bytes.  Every shell cell must be non-FLUID (else ST_EUNSUPPORTED).
+ * f_src is SCRATCH (ping-pong partner).  T = 0 copies.
+ */
+int lbm_d3q19_run(st_plan* plan, void* f_src, void* f_dst, double omega, int T,
+                  const uint8_t* flags);
+
+/* st_destroy — free the plan (NULL-safe).  Waits for its stream first. */
+void st_destroy(st_plan* plan);
+
+/* Thread-local description of the last error ("" if none). */
+const char* st_last_error(void);
+
+/* Thread-local ST_E* code of the last error (ST_OK if none); lets callers of
+ * st_plan_create (which returns NULL) see why. */
+int st_last_status(void);
+
+/* ---- optional setters / queries ------------------------------------------ */
+
+/* Run on this cudaStream_t (default: a plan-owned non-blocking stream). */
+int st_plan_set_stream(st_plan* plan, void* cuda_stream);
+
+/* Moving-lid velocity for LID cells (default (0.05, 0, 0)). */
+int st_plan_set_lbm_lid(st_plan* plan, double ux, double uy, double uz);
+
+/* 1: bit-exact kernels (no FMA contraction, oracle operation order). */
+int st_plan_set_bitexact(st_plan* plan, int on);
+
+/* Waits for the plan stream; returns ST_ECUDA for deferred device faults. */
+int st_plan_sync(st_plan* plan);
+
+/* Z-slab distribution (§8(e)): rank owns planes [z0, z0+nz_local) of the
+ * global grid (remainder planes go one each to the first ranks).  The
+ * 128-byte NCCL unique id comes from rank 0 (broadcast by the caller).
+ * nranks == 1 switches distribution off. */
+int st_plan_set_dist(st_plan* plan, const void* nccl_unique_id, int rank, int nranks);
+
+/* Loopback distribution on one device (testing): P virtual slabs, ghosts
+ * copied with cudaMemcpyAsync instead of NCCL; result identical to P = 1. */
+int st_plan_set_loopback_slabs(st_plan* plan, int nslabs);
+
+/* g = dim_T ghost planes per side of each slab in distributed mode (R = 1). */
+int st_plan_ghost_planes(const st_plan* plan);
+
+/* Local slab extent of this rank: first global plane and plane count. */
+int st_plan_local_slab(const st_plan* plan, int* z0, int* nz_local);
+
+/* Planner decisions, for logging/bench: tile TX x TY (loaded, incl. halo),
+ * output tile W_x x W_y, number of XY tiles, persistent CTAs, kernel variant. */
+typedef struct {
+    int tile_x, tile_y;     /* loaded XY sub-plane (dim_X, dim_Y of eq. (1))   */
+    int out_x, out_y;       /* written region per tile (dim - 2*R*dim_T) */
+    int tiles_x, tiles_y;   /* XY tiles covering the plane                      */
+    int ctas;               /* persistent CTAs launched per sweep               */
+    int threads;            /* threads per CTA                                  */
+    int smem_bytes;         /* dynamic shared memory per CTA                    */
+    double kappa;           /* eq. (2) analog: computed / useful points         */
+    int kernel;             /* internal variant id                               */
+    int dim_t_sweep;        /* deepest sweep actually run (<= dim_T, see above)  */
+} st_plan_info;
+int st_plan_get_info(const st_plan* plan, int lbm, st_plan_info* info);
+
+/* Number of kernel launches the last run enqueued (bench accounting). */
+int st_plan_last_launches(const st_plan* plan);
+
+/*
+ * Blocking-parameter model of §V-C (host-only, no device needed):
+ *   eq. (1)  E*(2R+2)*dim_T*dim_X*dim_Y <= C
+ *   eq. (2)  kappa = ((1-2R dim_T/dim_X)(1-2R dim_T/dim_Y))^-1
+ *   eq. (3)  dim_T >= eta = ceil(gamma/Gamma)
+ *   eq. (4)  dim_X = dim_Y = floor(sqrt(C/(E*(2R+2)*eta)))
+ * st_blocking_model fills eta, the eq. (4) real bound (before floor) and
+ * kappa for the given dim (dim <= 0: use the eq. (4) floor).
+ */
+typedef struct {
+    int eta;
+    double dim_bound;   /* sqrt(C/(E(2R+2)eta)) */
+    int dim;            /* tile side used for kappa */
+    double kappa;
+} st_blocking;
+int st_blocking_model(double C_bytes, double E_bytes, int R, double gamma, double Gamma,
+                      int dim_T, int dim, st_blocking* out);
+
+/* Paper's Fig. 3 buffer schedule (R, dim_T): at round r (0-based), level t'
+ * (0..dim_T) handles plane z = r - 2*R*t' in buffer slot
+ * z mod (2R+2); returns the step number S (1-based, chronological as in
+ * Fig. 3(a)) or 0 if level t' is idle in that round. */
+int st_fig3_step(int R, int dim_T, int round, int level, int* z, int* slot);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ST35D_H */

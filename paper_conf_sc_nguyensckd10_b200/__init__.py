@@ -1,0 +1,251 @@
+"""paper_conf_sc_nguyensckd10_b200 — thin Python binding of libst35d.so.
+
+Argument marshalling only: every step of the sweep runs in the library's
+sm_100a kernels (include/st35d.h).  Names mirror the C ABI:
+st_plan_create, st7_run, lbm_d3q19_run, st_destroy, ...
+
+Buffers may be torch CUDA tensors (the fast path: the call enqueues kernels
+on the plan stream and returns), or host numpy arrays / CPU tensors (the
+library stages them through device memory and synchronises).  There is no
+CPU fallback: without the built library or a CUDA device the calls raise.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libst35d.so")
+
+ST_F32, ST_F64 = 0, 1
+ST_OK, ST_EINVAL, ST_ENOMEM, ST_ECUDA, ST_ENCCL, ST_EUNSUPPORTED = 0, -1, -2, -3, -4, -5
+ST_FLUID, ST_WALL, ST_LID = 0, 1, 2
+ST_MAX_DIM_T = 8
+_ERRNAMES = {-1: "ST_EINVAL", -2: "ST_ENOMEM", -3: "ST_ECUDA", -4: "ST_ENCCL", -5: "ST_EUNSUPPORTED"}
+
+
+class StError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"{_ERRNAMES.get(code, code)}: {msg}")
+        self.code = code
+
+
+class st_plan_info(ctypes.Structure):
+    _fields_ = [("tile_x", ctypes.c_int), ("tile_y", ctypes.c_int), ("out_x", ctypes.c_int),
+                ("out_y", ctypes.c_int), ("tiles_x", ctypes.c_int), ("tiles_y", ctypes.c_int),
+                ("ctas", ctypes.c_int), ("threads", ctypes.c_int), ("smem_bytes", ctypes.c_int),
+                ("kappa", ctypes.c_double), ("kernel", ctypes.c_int), ("dim_t_sweep", ctypes.c_int)]
+
+
+class st_blocking(ctypes.Structure):
+    _fields_ = [("eta", ctypes.c_int), ("dim_bound", ctypes.c_double), ("dim", ctypes.c_int),
+                ("kappa", ctypes.c_double)]
+
+
+_lib = None
+
+EXPORTS = ["st_plan_create", "st7_run", "lbm_d3q19_run", "st_destroy", "st_last_error", "st_last_status",
+           "st_plan_set_stream", "st_plan_set_lbm_lid", "st_plan_set_bitexact", "st_plan_sync",
+           "st_plan_set_dist", "st_plan_set_loopback_slabs", "st_plan_ghost_planes", "st_plan_local_slab",
+           "st_plan_get_info", "st_plan_last_launches", "st_blocking_model", "st_fig3_step"]
+
+
+def lib() -> ctypes.CDLL:
+    """Load libst35d.so (raises if it was not built: there is no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} missing: run `python -c 'import __graft_entry__ as g; g.build()'`")
+    L = ctypes.CDLL(LIB_PATH)
+    P, I, D = ctypes.c_void_p, ctypes.c_int, ctypes.c_double
+    sig = {
+        "st_plan_create": ([I, I, I, I, I], P),
+        "st7_run": ([P, P, P, D, D, I], I),
+        "lbm_d3q19_run": ([P, P, P, D, I, P], I),
+        "st_destroy": ([P], None),
+        "st_last_error": ([], ctypes.c_char_p),
+        "st_last_status": ([], I),
+        "st_plan_set_stream": ([P, P], I),
+        "st_plan_set_lbm_lid": ([P, D, D, D], I),
+        "st_plan_set_bitexact": ([P, I], I),
+        "st_plan_sync": ([P], I),
+        "st_plan_set_dist": ([P, P, I, I], I),
+        "st_plan_set_loopback_slabs": ([P, I], I),
+        "st_plan_ghost_planes": ([P], I),
+        "st_plan_local_slab": ([P, ctypes.POINTER(I), ctypes.POINTER(I)], I),
+        "st_plan_get_info": ([P, I, ctypes.POINTER(st_plan_info)], I),
+        "st_plan_last_launches": ([P], I),
+        "st_blocking_model": ([D, D, I, D, D, I, I, ctypes.POINTER(st_blocking)], I),
+        "st_fig3_step": ([I, I, I, I, ctypes.POINTER(I), ctypes.POINTER(I)], I),
+    }
+    for name, (args, res) in sig.items():
+        fn = getattr(L, name)
+        fn.argtypes = args
+        fn.restype = res
+    _lib = L
+    return L
+
+
+def st_last_error() -> str:
+    return lib().st_last_error().decode()
+
+
+def _check(rc: int) -> int:
+    if rc < 0:
+        raise StError(rc, st_last_error())
+    return rc
+
+
+def _ptr(buf) -> int:
+    """device or host address of a torch tensor / numpy array / int."""
+    if buf is None:
+        return 0
+    if isinstance(buf, int):
+        return buf
+    if hasattr(buf, "data_ptr"):
+        if not buf.is_contiguous():
+            raise ValueError("tensor must be contiguous")
+        return buf.data_ptr()
+    if hasattr(buf, "ctypes"):
+        if not buf.flags["C_CONTIGUOUS"]:
+            raise ValueError("array must be C-contiguous")
+        return buf.ctypes.data
+    raise TypeError(type(buf))
+
+
+def st_plan_create(nx: int, ny: int, nz: int, dtype: int, dim_T: int) -> int:
+    h = lib().st_plan_create(nx, ny, nz, dtype, dim_T)
+    if not h:
+        raise StError(lib().st_last_status() or ST_EINVAL, st_last_error())
+    return h
+
+
+def st7_run(plan: int, inp, out, alpha: float, beta: float, T: int) -> int:
+    return _check(lib().st7_run(plan, _ptr(inp), _ptr(out), alpha, beta, T))
+
+
+def lbm_d3q19_run(plan: int, f_src, f_dst, omega: float, T: int, flags) -> int:
+    return _check(lib().lbm_d3q19_run(plan, _ptr(f_src), _ptr(f_dst), omega, T, _ptr(flags)))
+
+
+def st_destroy(plan: int) -> None:
+    if plan:
+        lib().st_destroy(plan)
+
+
+def st_plan_set_stream(plan: int, stream) -> int:
+    s = stream if isinstance(stream, int) else getattr(stream, "cuda_stream", 0)
+    return _check(lib().st_plan_set_stream(plan, s))
+
+
+def st_plan_set_lbm_lid(plan: int, ux: float, uy: float, uz: float) -> int:
+    return _check(lib().st_plan_set_lbm_lid(plan, ux, uy, uz))
+
+
+def st_plan_set_bitexact(plan: int, on: bool) -> int:
+    return _check(lib().st_plan_set_bitexact(plan, 1 if on else 0))
+
+
+def st_plan_sync(plan: int) -> int:
+    return _check(lib().st_plan_sync(plan))
+
+
+def st_plan_set_dist(plan: int, unique_id: bytes, rank: int, nranks: int) -> int:
+    buf = ctypes.create_string_buffer(bytes(unique_id), 128)
+    return _check(lib().st_plan_set_dist(plan, ctypes.addressof(buf), rank, nranks))
+
+
+def st_plan_set_loopback_slabs(plan: int, nslabs: int) -> int:
+    return _check(lib().st_plan_set_loopback_slabs(plan, nslabs))
+
+
+def st_plan_ghost_planes(plan: int) -> int:
+    return _check(lib().st_plan_ghost_planes(plan))
+
+
+def st_plan_local_slab(plan: int):
+    z0, n = ctypes.c_int(), ctypes.c_int()
+    _check(lib().st_plan_local_slab(plan, ctypes.byref(z0), ctypes.byref(n)))
+    return z0.value, n.value
+
+
+def st_plan_get_info(plan: int, lbm: bool = False) -> dict:
+    info = st_plan_info()
+    _check(lib().st_plan_get_info(plan, 1 if lbm else 0, ctypes.byref(info)))
+    return {k: getattr(info, k) for k, _ in st_plan_info._fields_}
+
+
+def st_plan_last_launches(plan: int) -> int:
+    return _check(lib().st_plan_last_launches(plan))
+
+
+def st_blocking_model(C_bytes: float, E_bytes: float, R: int, gamma: float, Gamma: float,
+                      dim_T: int = 0, dim: int = 0) -> dict:
+    out = st_blocking()
+    _check(lib().st_blocking_model(C_bytes, E_bytes, R, gamma, Gamma, dim_T, dim, ctypes.byref(out)))
+    return {k: getattr(out, k) for k, _ in st_blocking._fields_}
+
+
+def st_fig3_step(R: int, dim_T: int, rnd: int, level: int):
+    z, s = ctypes.c_int(), ctypes.c_int()
+    step = _check(lib().st_fig3_step(R, dim_T, rnd, level, ctypes.byref(z), ctypes.byref(s)))
+    return step, z.value, s.value
+
+
+def dtype_code(dtype) -> int:
+    name = str(dtype)
+    if "float32" in name:
+        return ST_F32
+    if "float64" in name:
+        return ST_F64
+    raise ValueError(f"unsupported dtype {dtype}")
+
+
+class Plan:
+    """RAII wrapper: ``with Plan(nx, ny, nz, dtype, dim_T) as p: p.st7(a, b, ...)``."""
+
+    def __init__(self, nx: int, ny: int, nz: int, dtype, dim_T: int):
+        self.h = st_plan_create(nx, ny, nz, dtype if isinstance(dtype, int) else dtype_code(dtype), dim_T)
+        self.shape = (nz, ny, nx)
+
+    def st7(self, inp, out, alpha: float, beta: float, T: int) -> None:
+        st7_run(self.h, inp, out, alpha, beta, T)
+
+    def lbm(self, f_src, f_dst, omega: float, T: int, flags) -> None:
+        lbm_d3q19_run(self.h, f_src, f_dst, omega, T, flags)
+
+    def set_stream(self, stream) -> None:
+        st_plan_set_stream(self.h, stream)
+
+    def set_bitexact(self, on: bool) -> None:
+        st_plan_set_bitexact(self.h, on)
+
+    def set_lid(self, ux: float, uy: float, uz: float) -> None:
+        st_plan_set_lbm_lid(self.h, ux, uy, uz)
+
+    def sync(self) -> None:
+        st_plan_sync(self.h)
+
+    def info(self, lbm: bool = False) -> dict:
+        return st_plan_get_info(self.h, lbm)
+
+    def last_launches(self) -> int:
+        return st_plan_last_launches(self.h)
+
+    def close(self) -> None:
+        if self.h:
+            st_destroy(self.h)
+            self.h = 0
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

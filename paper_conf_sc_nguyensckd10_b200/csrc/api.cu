@@ -1,0 +1,536 @@
+// api.cu — the C ABI (include/st35d.h): plan, planner, sweep driver,
+// TMA descriptors, host-pointer staging.  No torch types cross this boundary.
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <string>
+#include <vector>
+#include <algorithm>
+#include <cudaTypedefs.h>
+
+#include "../../include/st35d.h"
+#include "launch.h"
+#include "dist.h"
+
+using namespace st35d;
+
+// ----------------------------------------------------------------------------
+// errors
+// ----------------------------------------------------------------------------
+static thread_local std::string g_err;
+static thread_local int g_code = 0;
+
+static int fail(int code, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    g_code = code;
+    return code;
+}
+#define CUDA_TRY(x)                                                                          \
+    do {                                                                                     \
+        cudaError_t e_ = (x);                                                                \
+        if (e_ != cudaSuccess) return fail(ST_ECUDA, "%s: %s (%s:%d)", #x, cudaGetErrorString(e_), __FILE__, __LINE__); \
+    } while (0)
+
+extern "C" const char* st_last_error(void) { return g_err.c_str(); }
+extern "C" int st_last_status(void) { return g_code; }
+
+// ----------------------------------------------------------------------------
+// TMA descriptor encoding through the driver entry point (no -lcuda needed)
+// ----------------------------------------------------------------------------
+static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    if (!fn) {
+        void* p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+    }
+    return fn;
+}
+
+static int encode_3d(CUtensorMap* map, const void* base, st_dtype dt, int nx, int ny, int nz, int bx, int by) {
+    auto enc = get_encode();
+    if (!enc) return fail(ST_ECUDA, "cuTensorMapEncodeTiled unavailable");
+    const size_t E = dt == ST_F32 ? 4 : 8;
+    cuuint64_t dims[3] = {(cuuint64_t)nx, (cuuint64_t)ny, (cuuint64_t)nz};
+    cuuint64_t strides[2] = {(cuuint64_t)nx * E, (cuuint64_t)nx * ny * E};
+    cuuint32_t box[3] = {(cuuint32_t)bx, (cuuint32_t)by, 1};
+    cuuint32_t es[3] = {1, 1, 1};
+    CUresult r = enc(map, dt == ST_F32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3,
+                     const_cast<void*>(base), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                     CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return fail(ST_ECUDA, "cuTensorMapEncodeTiled failed (%d) box %dx%d", (int)r, bx, by);
+    return ST_OK;
+}
+
+// ----------------------------------------------------------------------------
+// plan
+// ----------------------------------------------------------------------------
+struct Geo7 {
+    int d = 0, VY = 0, NTX = 0, VX = 0, TX = 0, NTY = 0, TY = 0;
+    int hx = 0, wx = 0, wy = 0, tiles_x = 0, tiles_y = 0, threads = 0, grid = 0;
+    size_t smem = 0;
+    double kappa = 0;
+    St7LaunchFn fn = nullptr;
+};
+
+struct st_plan {
+    int nx, ny, nz;
+    st_dtype dtype;
+    int dimT;
+    int dimK = 0;      // deepest sweep the 7-point kernels can tile (<= dimT)
+    int dev = 0, sms = 0;
+    size_t smem_optin = 0;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    bool exact = false;
+    double lid[3] = {0.05, 0.0, 0.0};
+    int launches = 0;
+    // host-pointer staging
+    void* hbuf[2] = {nullptr, nullptr};
+    size_t hbuf_bytes = 0;
+    uint8_t* hflags = nullptr;
+    size_t hflags_bytes = 0;
+    int* d_count = nullptr;
+    int* h_count = nullptr;
+    const void* flags_checked = nullptr;
+    // distribution (Z slabs)
+    Dist dist;
+    std::map<int, Geo7> geo7;  // by depth
+};
+
+static size_t esize(st_dtype d) { return d == ST_F32 ? 4 : 8; }
+
+static int vy_for(st_dtype dt, int d) {
+    // register budget of the (D, VY) instantiations (ptxas -v: no spills)
+    if (dt == ST_F32) return d <= 4 ? 4 : 2;
+    return d <= 2 ? 4 : 2;
+}
+
+static St7LaunchFn lookup7(st_dtype dt, bool exact, int d, int vy) {
+    if (dt == ST_F32) return exact ? st7_lookup_f32_exact(d, vy) : st7_lookup_f32_fast(d, vy);
+    return exact ? st7_lookup_f64_exact(d, vy) : st7_lookup_f64_fast(d, vy);
+}
+
+static size_t smem7(const Geo7& g, st_dtype dt) {
+    return (size_t)ST7_RING * g.TX * g.TY * esize(dt) + (size_t)(g.d > 1 ? g.d - 1 : 0) * 4 * g.threads * 16 +
+           ST7_RING * 8;
+}
+
+// Planner for one sweep depth d over an nx x ny plane with nzo output planes:
+// eq. (1) analog (on-chip bytes of one SM: register file for the Z window,
+// shared memory for the TMA ring and the Y exchange), then the XY tile that
+// minimises computed points per plane (halo + ragged last tile), then a
+// persistent grid of one CTA per SM with equal (tile, z) volume per CTA.
+static int plan7(st_plan* p, int d, int nzo, Geo7& g) {
+    g.d = d;
+    g.VX = p->dtype == ST_F32 ? 4 : 2;
+    g.NTX = p->dtype == ST_F32 ? 16 : 32;
+    g.TX = g.NTX * g.VX;
+    g.VY = vy_for(p->dtype, d);
+    g.hx = (d + g.VX - 1) / g.VX * g.VX;
+    g.wx = (g.TX - g.hx - d) & ~(g.VX - 1);
+    if (g.wx < g.VX) return fail(ST_EUNSUPPORTED, "dim_T %d too deep for a %d-wide tile", d, g.TX);
+    g.tiles_x = (p->nx + g.wx - 1) / g.wx;
+    const int ntymax = ST7_MAXT / g.NTX;
+    long best = -1;
+    for (int nty = 2; nty <= ntymax; ++nty) {
+        Geo7 c = g;
+        c.NTY = nty;
+        c.TY = nty * c.VY;
+        c.threads = c.NTX * nty;
+        c.wy = c.TY - 2 * d;
+        if (c.wy < 1) continue;
+        c.tiles_y = (p->ny + c.wy - 1) / c.wy;
+        c.smem = smem7(c, p->dtype);
+        if (c.smem > p->smem_optin) continue;
+        long cost = (long)c.tiles_y * c.TY;
+        if (best < 0 || cost < best || (cost == best && c.TY > g.TY)) {
+            best = cost;
+            g = c;
+        }
+    }
+    if (best < 0) return fail(ST_EUNSUPPORTED, "no tile fits dim_T %d", d);
+    const long long work = (long long)g.tiles_x * g.tiles_y * nzo;
+    g.grid = (int)std::min<long long>(p->sms, std::max<long long>(work, 1));
+    g.kappa = (double)g.tiles_x * g.TX * g.tiles_y * g.TY / ((double)p->nx * p->ny);
+    g.fn = lookup7(p->dtype, p->exact, d, g.VY);
+    if (!g.fn) return fail(ST_EUNSUPPORTED, "no kernel for dim_T %d", d);
+    return ST_OK;
+}
+
+static int get_geo7(st_plan* p, int d, int nzo, Geo7*& out) {
+    auto it = p->geo7.find(d);
+    if (it == p->geo7.end() || it->second.fn != lookup7(p->dtype, p->exact, d, it->second.VY)) {
+        Geo7 g;
+        int rc = plan7(p, d, nzo, g);
+        if (rc) return rc;
+        it = p->geo7.insert_or_assign(d, g).first;
+    }
+    out = &it->second;
+    // grid depends on the output-plane count of the call
+    const long long work = (long long)out->tiles_x * out->tiles_y * nzo;
+    out->grid = (int)std::min<long long>(p->sms, std::max<long long>(work, 1));
+    return ST_OK;
+}
+
+extern "C" st_plan* st_plan_create(int nx, int ny, int nz, st_dtype dtype, int dim_T) {
+    if (nx < 3 || ny < 3 || nz < 3) { fail(ST_EINVAL, "grid %dx%dx%d: every extent must be >= 3", nx, ny, nz); return nullptr; }
+    if (dtype != ST_F32 && dtype != ST_F64) { fail(ST_EINVAL, "dtype %d", (int)dtype); return nullptr; }
+    if (dim_T < 1 || dim_T > ST_MAX_DIM_T) { fail(ST_EINVAL, "dim_T %d not in [1, %d]", dim_T, ST_MAX_DIM_T); return nullptr; }
+    if (((size_t)nx * esize(dtype)) % 16 != 0) {
+        fail(ST_EUNSUPPORTED, "nx*sizeof(dtype) = %zu is not a multiple of 16 bytes (TMA row pitch)",
+             (size_t)nx * esize(dtype));
+        return nullptr;
+    }
+    int dev = 0, cnt = 0;
+    if (cudaGetDeviceCount(&cnt) != cudaSuccess || cnt == 0) { fail(ST_ECUDA, "no CUDA device"); cudaGetLastError(); return nullptr; }
+    cudaGetDevice(&dev);
+    cudaDeviceProp prop;
+    if (cudaGetDeviceProperties(&prop, dev) != cudaSuccess) { fail(ST_ECUDA, "cudaGetDeviceProperties"); return nullptr; }
+    if (prop.major < 10) { fail(ST_EUNSUPPORTED, "needs sm_100a (found sm_%d%d)", prop.major, prop.minor); return nullptr; }
+    st_plan* p = new st_plan();
+    p->nx = nx; p->ny = ny; p->nz = nz; p->dtype = dtype; p->dimT = dim_T;
+    p->dev = dev;
+    p->sms = prop.multiProcessorCount;
+    p->smem_optin = prop.sharedMemPerBlockOptin;
+    if (cudaStreamCreateWithFlags(&p->stream, cudaStreamNonBlocking) != cudaSuccess) {
+        fail(ST_ECUDA, "stream create"); delete p; return nullptr;
+    }
+    p->own_stream = true;
+    if (cudaMalloc(&p->d_count, sizeof(int)) != cudaSuccess || cudaMallocHost(&p->h_count, sizeof(int)) != cudaSuccess) {
+        fail(ST_ENOMEM, "scratch"); st_destroy(p); return nullptr;
+    }
+    p->dist.init_single(nz);
+    // deepest 7-point sweep that tiles on one SM (f64 at dim_T 7-8 does not:
+    // those plans run sweeps of depth dimK < dim_T; results are identical)
+    Geo7* g = nullptr;
+    for (int d = dim_T; d >= 1; --d)
+        if (get_geo7(p, d, nz, g) == ST_OK) { p->dimK = d; break; }
+    if (!p->dimK) { st_destroy(p); return nullptr; }
+    g_err.clear();
+    g_code = 0;
+    return p;
+}
+
+extern "C" void st_destroy(st_plan* p) {
+    if (!p) return;
+    if (p->stream) cudaStreamSynchronize(p->stream);
+    p->dist.destroy();
+    for (void* b : p->hbuf) if (b) cudaFree(b);
+    if (p->hflags) cudaFree(p->hflags);
+    if (p->d_count) cudaFree(p->d_count);
+    if (p->h_count) cudaFreeHost(p->h_count);
+    if (p->own_stream && p->stream) cudaStreamDestroy(p->stream);
+    delete p;
+}
+
+extern "C" int st_plan_set_stream(st_plan* p, void* s) {
+    if (!p) return fail(ST_EINVAL, "NULL plan");
+    if (p->own_stream && p->stream) { cudaStreamSynchronize(p->stream); cudaStreamDestroy(p->stream); }
+    p->stream = static_cast<cudaStream_t>(s);
+    p->own_stream = false;
+    return ST_OK;
+}
+
+extern "C" int st_plan_set_lbm_lid(st_plan* p, double ux, double uy, double uz) {
+    if (!p) return fail(ST_EINVAL, "NULL plan");
+    p->lid[0] = ux; p->lid[1] = uy; p->lid[2] = uz;
+    return ST_OK;
+}
+
+extern "C" int st_plan_set_bitexact(st_plan* p, int on) {
+    if (!p) return fail(ST_EINVAL, "NULL plan");
+    p->exact = on != 0;
+    return ST_OK;
+}
+
+extern "C" int st_plan_sync(st_plan* p) {
+    if (!p) return fail(ST_EINVAL, "NULL plan");
+    CUDA_TRY(cudaStreamSynchronize(p->stream));
+    CUDA_TRY(cudaGetLastError());
+    return ST_OK;
+}
+
+extern "C" int st_plan_ghost_planes(const st_plan* p) { return p ? p->dimT : ST_EINVAL; }
+
+extern "C" int st_plan_local_slab(const st_plan* p, int* z0, int* nzl) {
+    if (!p) return fail(ST_EINVAL, "NULL plan");
+    if (z0) *z0 = p->dist.z0;
+    if (nzl) *nzl = p->dist.nzl;
+    return ST_OK;
+}
+
+extern "C" int st_plan_last_launches(const st_plan* p) { return p ? p->launches : ST_EINVAL; }
+
+extern "C" int st_plan_get_info(const st_plan* p, int lbm, st_plan_info* info) {
+    if (!p || !info) return fail(ST_EINVAL, "NULL argument");
+    memset(info, 0, sizeof *info);
+    if (lbm) {
+        info->tile_x = p->nx; info->tile_y = p->ny; info->out_x = p->nx; info->out_y = p->ny;
+        info->tiles_x = info->tiles_y = 1; info->ctas = p->sms * 8; info->threads = 256; info->kappa = 1.0;
+        info->kernel = 100;
+        info->dim_t_sweep = 1;
+        return ST_OK;
+    }
+    auto it = p->geo7.find(p->dimK);
+    if (it == p->geo7.end()) return fail(ST_EINVAL, "no plan for dim_T");
+    const Geo7& g = it->second;
+    info->tile_x = g.TX; info->tile_y = g.TY; info->out_x = g.wx; info->out_y = g.wy;
+    info->tiles_x = g.tiles_x; info->tiles_y = g.tiles_y; info->ctas = g.grid; info->threads = g.threads;
+    info->smem_bytes = (int)g.smem; info->kappa = g.kappa; info->kernel = g.VY;
+    info->dim_t_sweep = p->dimK;
+    return ST_OK;
+}
+
+// ----------------------------------------------------------------------------
+// helpers
+// ----------------------------------------------------------------------------
+static int ptr_kind(const void* ptr) {  // 1 device, 0 host, -1 error
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, ptr) != cudaSuccess) { cudaGetLastError(); return 0; }
+    return (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) ? 1 : 0;
+}
+
+static int ensure_hbuf(st_plan* p, size_t bytes) {
+    if (p->hbuf_bytes >= bytes) return ST_OK;
+    for (void*& b : p->hbuf) { if (b) cudaFree(b); b = nullptr; }
+    p->hbuf_bytes = 0;
+    for (void*& b : p->hbuf)
+        if (cudaMalloc(&b, bytes) != cudaSuccess) { cudaGetLastError(); return fail(ST_ENOMEM, "device staging %zu B", bytes); }
+    p->hbuf_bytes = bytes;
+    return ST_OK;
+}
+
+// depths of the sweeps: S = ceil(T/dim_T) sweeps, made odd so the result
+// lands in `out` (ping-pong); depths as equal as possible, each <= dim_T
+static std::vector<int> sweep_depths(int T, int D) {
+    std::vector<int> v;
+    if (T <= 0) return v;
+    int S = (T + D - 1) / D;
+    if (S % 2 == 0 && S < T) ++S;
+    const int q = T / S, rem = T % S;
+    for (int s = 0; s < S; ++s) v.push_back(q + (s < rem ? 1 : 0));
+    return v;
+}
+
+static bool overlap(const void* a, const void* b, size_t n) {
+    auto x = reinterpret_cast<uintptr_t>(a), y = reinterpret_cast<uintptr_t>(b);
+    return x < y + n && y < x + n;
+}
+
+// ----------------------------------------------------------------------------
+// 7-point
+// ----------------------------------------------------------------------------
+static int launch7(st_plan* p, const void* src, void* dst, int d, double alpha, double beta, const SlabView& sv) {
+    Geo7* g = nullptr;
+    int rc = get_geo7(p, d, sv.zb - sv.za, g);
+    if (rc) return rc;
+    CUtensorMap map;
+    rc = encode_3d(&map, src, p->dtype, p->nx, p->ny, sv.nzb, g->TX, g->TY);
+    if (rc) return rc;
+    St7Params prm{};
+    prm.out = dst;
+    prm.nx = p->nx; prm.ny = p->ny; prm.nzb = sv.nzb; prm.zbase = sv.zbase; prm.nzg = p->nz;
+    prm.za = sv.za; prm.zb = sv.zb;
+    prm.tiles_x = g->tiles_x; prm.ntiles = g->tiles_x * g->tiles_y;
+    prm.wx = g->wx; prm.wy = g->wy; prm.hx = g->hx;
+    prm.work = (long long)prm.ntiles * (sv.zb - sv.za);
+    prm.alpha = alpha; prm.beta = beta;
+    if (prm.work <= 0) return ST_OK;
+    cudaError_t e = g->fn(&map, prm, g->grid, g->threads, g->smem, sv.stream ? sv.stream : p->stream);
+    if (e != cudaSuccess) return fail(ST_ECUDA, "st7 launch (d=%d): %s", d, cudaGetErrorString(e));
+    ++p->launches;
+    return ST_OK;
+}
+
+static int run7_device(st_plan* p, const void* in, void* out, double alpha, double beta, int T) {
+    const size_t n = (size_t)p->nx * p->ny * p->dist.nzb * esize(p->dtype);
+    p->launches = 0;
+    if (T == 0) {
+        CUDA_TRY(cudaMemcpyAsync(out, in, n, cudaMemcpyDeviceToDevice, p->stream));
+        return ST_OK;
+    }
+    std::vector<int> ds = sweep_depths(T, p->dimK);
+    const void* src = in;
+    void* dst = out;
+    void* bufs[2] = {const_cast<void*>(in), out};
+    for (size_t s = 0; s < ds.size(); ++s) {
+        int rc = p->dist.sweep(p->stream, ds[s], src, dst, esize(p->dtype), (size_t)p->nx * p->ny,
+                               [&](const void* a, void* b, const SlabView& sv) {
+                                   return launch7(p, a, b, ds[s], alpha, beta, sv);
+                               });
+        if (rc) return rc;
+        src = bufs[(s + 1) % 2];
+        dst = bufs[s % 2];
+    }
+    if (ds.size() % 2 == 0)  // only when dim_T = 1 and T even: result is in `in`
+        CUDA_TRY(cudaMemcpyAsync(out, in, n, cudaMemcpyDeviceToDevice, p->stream));
+    CUDA_TRY(cudaGetLastError());
+    return ST_OK;
+}
+
+extern "C" int st7_run(st_plan* p, const void* in, void* out, double alpha, double beta, int T) {
+    if (!p) return fail(ST_EINVAL, "NULL plan");
+    if (!in || !out) return fail(ST_EINVAL, "NULL grid pointer");
+    if (T < 0) return fail(ST_EINVAL, "T = %d < 0", T);
+    const size_t n = (size_t)p->nx * p->ny * p->dist.nzb * esize(p->dtype);
+    if (overlap(in, out, n)) return fail(ST_EINVAL, "in and out overlap");
+    const int kin = ptr_kind(in), kout = ptr_kind(out);
+    if (kin != kout) return fail(ST_EINVAL, "in and out must both be host or both be device pointers");
+    if (kin == 1) {
+        if ((reinterpret_cast<uintptr_t>(in) | reinterpret_cast<uintptr_t>(out)) & 15)
+            return fail(ST_EINVAL, "device grids must be 16-byte aligned");
+        return run7_device(p, in, out, alpha, beta, T);
+    }
+    // host pointers: stage through plan-owned device buffers, synchronous
+    int rc = ensure_hbuf(p, n);
+    if (rc) return rc;
+    CUDA_TRY(cudaMemcpyAsync(p->hbuf[0], in, n, cudaMemcpyHostToDevice, p->stream));
+    rc = run7_device(p, p->hbuf[0], p->hbuf[1], alpha, beta, T);
+    if (rc) return rc;
+    CUDA_TRY(cudaMemcpyAsync(out, p->hbuf[1], n, cudaMemcpyDeviceToHost, p->stream));
+    CUDA_TRY(cudaStreamSynchronize(p->stream));
+    return ST_OK;
+}
+
+// ----------------------------------------------------------------------------
+// LBM D3Q19
+// ----------------------------------------------------------------------------
+template <typename T>
+static void lid_coeffs(const double lid[3], double out[19]) {
+    static const int ex[19] = {0, 1, -1, 0, 0, 0, 0, 1, -1, 1, -1, 1, -1, 1, -1, 0, 0, 0, 0};
+    static const int ey[19] = {0, 0, 0, 1, -1, 0, 0, 1, -1, -1, 1, 0, 0, 0, 0, 1, -1, 1, -1};
+    static const int ez[19] = {0, 0, 0, 0, 0, 1, -1, 0, 0, 0, 0, 1, -1, -1, 1, 1, -1, -1, 1};
+    const T u[3] = {(T)lid[0], (T)lid[1], (T)lid[2]};
+    for (int i = 0; i < 19; ++i) {
+        const int e[3] = {ex[i], ey[i], ez[i]};
+        T eu = 0;
+        bool first = true;
+        for (int a = 0; a < 3; ++a) {
+            if (!e[a]) continue;
+            T v = e[a] > 0 ? u[a] : -u[a];
+            eu = first ? v : (T)(eu + v);
+            first = false;
+        }
+        const T w = (T)1 / (T)(i == 0 ? 3 : (i <= 6 ? 18 : 36));
+        const T sixw = (T)((T)6 * w);
+        out[i] = (double)(T)(sixw * eu);
+    }
+}
+
+static int launch_lbm(st_plan* p, const void* src, void* dst, const uint8_t* flags, double omega,
+                      const SlabView& sv) {
+    LbmParams prm{};
+    prm.nx = p->nx; prm.ny = p->ny; prm.nzb = sv.nzb; prm.zbase = sv.zbase; prm.nzg = p->nz;
+    prm.za = sv.za; prm.zb = sv.zb;
+    prm.omega = omega;
+    if (p->dtype == ST_F32) lid_coeffs<float>(p->lid, prm.lidc);
+    else lid_coeffs<double>(p->lid, prm.lidc);
+    const long long cells = (long long)(sv.zb - sv.za) * p->nx * p->ny;
+    if (cells <= 0) return ST_OK;
+    const int grid = (int)std::min<long long>((cells + 255) / 256, (long long)p->sms * 16);
+    cudaError_t e = lbm_push_launch(p->dtype == ST_F32 ? 0 : 1, p->exact, src, dst, flags, prm, grid,
+                                    sv.stream ? sv.stream : p->stream);
+    if (e != cudaSuccess) return fail(ST_ECUDA, "lbm launch: %s", cudaGetErrorString(e));
+    ++p->launches;
+    return ST_OK;
+}
+
+static int check_shell(st_plan* p, const uint8_t* flags) {
+    if (p->flags_checked == flags) return ST_OK;
+    if (p->dist.nranks > 1) { p->flags_checked = flags; return ST_OK; }  // slab shells checked per rank
+    cudaError_t e = lbm_shell_check(flags, p->nx, p->ny, p->nz, p->d_count, p->stream);
+    if (e != cudaSuccess) return fail(ST_ECUDA, "shell check: %s", cudaGetErrorString(e));
+    CUDA_TRY(cudaMemcpyAsync(p->h_count, p->d_count, sizeof(int), cudaMemcpyDeviceToHost, p->stream));
+    CUDA_TRY(cudaStreamSynchronize(p->stream));
+    if (*p->h_count != 0)
+        return fail(ST_EUNSUPPORTED, "%d shell cells are FLUID; the GPU path needs a non-FLUID shell", *p->h_count);
+    p->flags_checked = flags;
+    return ST_OK;
+}
+
+static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T, const uint8_t* flags) {
+    const size_t n = 19 * (size_t)p->nx * p->ny * p->dist.nzb * esize(p->dtype);
+    p->launches = 0;
+    int rc = check_shell(p, flags);
+    if (rc) return rc;
+    if (T == 0) {
+        CUDA_TRY(cudaMemcpyAsync(fdst, fsrc, n, cudaMemcpyDeviceToDevice, p->stream));
+        return ST_OK;
+    }
+    // dim_T = 1 push sweeps (the on-chip multi-level LBM sweep is lbm_35d)
+    const void* src = fsrc;
+    void* dst = fdst;
+    void* bufs[2] = {fsrc, fdst};
+    const int S = T;
+    for (int s = 0; s < S; ++s) {
+        rc = p->dist.sweep(p->stream, 1, src, dst, 19 * esize(p->dtype), (size_t)p->nx * p->ny,
+                           [&](const void* a, void* b, const SlabView& sv) {
+                               return launch_lbm(p, a, b, flags + (sv.flags_off), omega, sv);
+                           });
+        if (rc) return rc;
+        src = bufs[(s + 1) % 2];
+        dst = bufs[s % 2];
+    }
+    if (S % 2 == 0) CUDA_TRY(cudaMemcpyAsync(fdst, fsrc, n, cudaMemcpyDeviceToDevice, p->stream));
+    CUDA_TRY(cudaGetLastError());
+    return ST_OK;
+}
+
+extern "C" int lbm_d3q19_run(st_plan* p, void* fsrc, void* fdst, double omega, int T, const uint8_t* flags) {
+    if (!p) return fail(ST_EINVAL, "NULL plan");
+    if (!fsrc || !fdst || !flags) return fail(ST_EINVAL, "NULL pointer");
+    if (T < 0) return fail(ST_EINVAL, "T = %d < 0", T);
+    if (!(omega >= 0.0 && omega < 2.0)) return fail(ST_EINVAL, "omega = %g not in [0, 2)", omega);
+    const size_t cells = (size_t)p->nx * p->ny * p->dist.nzb;
+    const size_t n = 19 * cells * esize(p->dtype);
+    if (overlap(fsrc, fdst, n)) return fail(ST_EINVAL, "f_src and f_dst overlap");
+    const int ks = ptr_kind(fsrc), kd = ptr_kind(fdst), kf = ptr_kind(flags);
+    if (ks != kd || ks != kf) return fail(ST_EINVAL, "f_src, f_dst and flags must all be host or all device");
+    if (ks == 1) {
+        if ((reinterpret_cast<uintptr_t>(fsrc) | reinterpret_cast<uintptr_t>(fdst)) & 15)
+            return fail(ST_EINVAL, "device lattices must be 16-byte aligned");
+        return runlbm_device(p, fsrc, fdst, omega, T, flags);
+    }
+    int rc = ensure_hbuf(p, n);
+    if (rc) return rc;
+    if (p->hflags_bytes < cells) {
+        if (p->hflags) cudaFree(p->hflags);
+        p->hflags = nullptr; p->hflags_bytes = 0;
+        if (cudaMalloc(&p->hflags, cells) != cudaSuccess) { cudaGetLastError(); return fail(ST_ENOMEM, "flags staging"); }
+        p->hflags_bytes = cells;
+    }
+    CUDA_TRY(cudaMemcpyAsync(p->hbuf[0], fsrc, n, cudaMemcpyHostToDevice, p->stream));
+    CUDA_TRY(cudaMemcpyAsync(p->hflags, flags, cells, cudaMemcpyHostToDevice, p->stream));
+    p->flags_checked = nullptr;  // staging buffer content changes per call
+    rc = runlbm_device(p, p->hbuf[0], p->hbuf[1], omega, T, p->hflags);
+    if (rc) return rc;
+    CUDA_TRY(cudaMemcpyAsync(fdst, p->hbuf[1], n, cudaMemcpyDeviceToHost, p->stream));
+    CUDA_TRY(cudaStreamSynchronize(p->stream));
+    return ST_OK;
+}
+
+// ----------------------------------------------------------------------------
+// distribution (Z slabs)
+// ----------------------------------------------------------------------------
+extern "C" int st_plan_set_dist(st_plan* p, const void* uid, int rank, int nranks) {
+    if (!p) return fail(ST_EINVAL, "NULL plan");
+    if (nranks == 1) { p->dist.init_single(p->nz); return ST_OK; }
+    (void)uid; (void)rank;
+    return fail(ST_EUNSUPPORTED, "distributed Z slabs not built yet");
+}
+
+extern "C" int st_plan_set_loopback_slabs(st_plan* p, int nslabs) {
+    if (!p) return fail(ST_EINVAL, "NULL plan");
+    if (nslabs == 1) { p->dist.init_single(p->nz); return ST_OK; }
+    return fail(ST_EUNSUPPORTED, "loopback slabs not built yet");
+}

@@ -1,0 +1,26 @@
+// launch.h — internal dispatch between the C-ABI (api.cu) and the kernel
+// instantiation units (st7_inst.cu compiled per dtype/mode, lbm_inst.cu).
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include "st7_kernel.cuh"
+#include "lbm_kernel.cuh"
+
+namespace st35d {
+
+using St7LaunchFn = cudaError_t (*)(const CUtensorMap* map, const St7Params& p, int grid, int threads,
+                                    size_t smem, cudaStream_t s);
+
+// returns nullptr if (D, VY) is not compiled
+St7LaunchFn st7_lookup_f32_fast(int D, int VY);
+St7LaunchFn st7_lookup_f32_exact(int D, int VY);
+St7LaunchFn st7_lookup_f64_fast(int D, int VY);
+St7LaunchFn st7_lookup_f64_exact(int D, int VY);
+
+cudaError_t lbm_push_launch(int dtype, bool exact, const void* src, void* dst, const uint8_t* flags,
+                            const LbmParams& p, int grid, cudaStream_t s);
+cudaError_t lbm_shell_check(const uint8_t* flags, int nx, int ny, int nz, int* d_count, cudaStream_t s);
+
+constexpr int ST7_MAXT = 256;
+
+}  // namespace st35d

@@ -1,0 +1,161 @@
+// lbm_kernel.cuh — D3Q19 lattice-Boltzmann step kernels for sm_100a.
+//
+// One step: read the 19 values and the flag of a cell,
+// collide (BGK, X9), propagate the 19 new values to the 18
+// neighbours and the cell itself; links into WALL cells bounce back, links
+// into LID cells bounce back with the Ladd correction; non-FLUID cells keep
+// their values.  The stored state is post-stream / pre-collision (X13).
+//
+// lbm_push_kernel (dim_T = 1 sweep): one thread per cell, SoA coalesced
+// loads of the 19 populations, collision in registers,
+// propagation as coalesced (x-shifted) stores — GPU stores do not
+// write-allocate, so the paper's 228 B/update is 153 B here (X12).
+//
+// The collision arithmetic follows the oracle's operation order (X20); in
+// bit-exact mode every operation is an explicitly rounded intrinsic, in the
+// default mode the compiler may contract products into FMAs.
+#pragma once
+#include "common.cuh"
+
+namespace st35d {
+
+struct LbmParams {
+    int nx, ny;
+    int nzb;          // planes in the local buffers
+    int zbase, nzg;   // global z of local plane 0, global nz
+    int za, zb;       // local planes updated [za, zb)
+    double omega;
+    double lidc[19];  // (6 w_i)(e_i . u_lid), computed on the host in the plan dtype
+};
+
+// velocity set (X10): 0; +x -x +y -y +z -z; edges 7..18
+__constant__ int8_t c_ex[19] = {0, 1, -1, 0, 0, 0, 0, 1, -1, 1, -1, 1, -1, 1, -1, 0, 0, 0, 0};
+__constant__ int8_t c_ey[19] = {0, 0, 0, 1, -1, 0, 0, 1, -1, -1, 1, 0, 0, 0, 0, 1, -1, 1, -1};
+__constant__ int8_t c_ez[19] = {0, 0, 0, 0, 0, 1, -1, 0, 0, 0, 0, 1, -1, -1, 1, 1, -1, -1, 1};
+
+template <int I> struct D3Q19 {
+    static constexpr int ex = (I == 1 || I == 7 || I == 9 || I == 11 || I == 13) ? 1
+                            : (I == 2 || I == 8 || I == 10 || I == 12 || I == 14) ? -1 : 0;
+    static constexpr int ey = (I == 3 || I == 7 || I == 10 || I == 15 || I == 17) ? 1
+                            : (I == 4 || I == 8 || I == 9 || I == 16 || I == 18) ? -1 : 0;
+    static constexpr int ez = (I == 5 || I == 11 || I == 14 || I == 15 || I == 18) ? 1
+                            : (I == 6 || I == 12 || I == 13 || I == 16 || I == 17) ? -1 : 0;
+    static constexpr int wden = I == 0 ? 3 : (I <= 6 ? 18 : 36);
+    static constexpr int opp = I == 0 ? 0 : ((I & 1) ? I + 1 : I - 1);
+};
+
+template <typename T, bool EXACT> struct Ar;
+template <bool E> struct Ar<float, E> {
+    static __device__ __forceinline__ float add(float a, float b) { return E ? __fadd_rn(a, b) : a + b; }
+    static __device__ __forceinline__ float sub(float a, float b) { return E ? __fsub_rn(a, b) : a - b; }
+    static __device__ __forceinline__ float mul(float a, float b) { return E ? __fmul_rn(a, b) : a * b; }
+    static __device__ __forceinline__ float div(float a, float b) { return __fdiv_rn(a, b); }
+};
+template <bool E> struct Ar<double, E> {
+    static __device__ __forceinline__ double add(double a, double b) { return E ? __dadd_rn(a, b) : a + b; }
+    static __device__ __forceinline__ double sub(double a, double b) { return E ? __dsub_rn(a, b) : a - b; }
+    static __device__ __forceinline__ double mul(double a, double b) { return E ? __dmul_rn(a, b) : a * b; }
+    static __device__ __forceinline__ double div(double a, double b) { return __ddiv_rn(a, b); }
+};
+
+// signed accumulation of e_a * f over the non-zero components, oracle order (X20)
+template <typename T, bool E, int A, int I = 0>
+__device__ __forceinline__ void jsum(const T (&f)[19], T& acc, bool& first) {
+    if constexpr (I < 19) {
+        constexpr int e = A == 0 ? D3Q19<I>::ex : (A == 1 ? D3Q19<I>::ey : D3Q19<I>::ez);
+        if constexpr (e != 0) {
+            if (first) { acc = e > 0 ? f[I] : -f[I]; first = false; }
+            else acc = e > 0 ? Ar<T, E>::add(acc, f[I]) : Ar<T, E>::sub(acc, f[I]);
+        }
+        jsum<T, E, A, I + 1>(f, acc, first);
+    }
+}
+
+template <typename T, bool E, int I>
+__device__ __forceinline__ T edotu(T ux, T uy, T uz) {
+    constexpr int ex = D3Q19<I>::ex, ey = D3Q19<I>::ey, ez = D3Q19<I>::ez;
+    T eu = T(0);
+    bool first = true;
+    if constexpr (ex != 0) { eu = ex > 0 ? ux : -ux; first = false; }
+    if constexpr (ey != 0) { T v = ey > 0 ? uy : -uy; eu = first ? v : Ar<T, E>::add(eu, v); first = false; }
+    if constexpr (ez != 0) { T v = ez > 0 ? uz : -uz; eu = first ? v : Ar<T, E>::add(eu, v); first = false; }
+    (void)first;
+    return eu;
+}
+
+// BGK collision of one cell in place: f <- f - omega (f - feq), oracle order.
+template <typename T, bool E>
+__device__ __forceinline__ void collide(T (&f)[19], T omega) {
+    using A = Ar<T, E>;
+    T rho = f[0];
+#pragma unroll
+    for (int i = 1; i < 19; ++i) rho = A::add(rho, f[i]);
+    T jx, jy, jz;
+    bool fx = true, fy = true, fz = true;
+    jsum<T, E, 0>(f, jx, fx);
+    jsum<T, E, 1>(f, jy, fy);
+    jsum<T, E, 2>(f, jz, fz);
+    const T ux = A::div(jx, rho), uy = A::div(jy, rho), uz = A::div(jz, rho);
+    T usq = A::add(A::mul(ux, ux), A::mul(uy, uy));
+    usq = A::add(usq, A::mul(uz, uz));
+    const T usq15 = A::mul(T(1.5), usq);
+    auto one = [&](auto Ic) {
+        constexpr int I = decltype(Ic)::value;
+        const T eu = edotu<T, E, I>(ux, uy, uz);
+        const T w = T(1) / T(D3Q19<I>::wden);
+        const T wr = A::mul(w, rho);
+        const T a = A::add(T(1), A::mul(T(3), eu));
+        const T c = A::mul(A::mul(T(4.5), eu), eu);
+        const T g = A::sub(A::add(a, c), usq15);
+        const T feq = A::mul(wr, g);
+        f[I] = A::sub(f[I], A::mul(omega, A::sub(f[I], feq)));
+    };
+    [&]<int... Is>(std::integer_sequence<int, Is...>) { (one(std::integral_constant<int, Is>{}), ...); }
+    (std::make_integer_sequence<int, 19>{});
+}
+
+// dim_T = 1: push form, one thread per cell, grid-stride over the updated planes.
+template <typename T, bool E>
+__global__ void __launch_bounds__(256)
+lbm_push_kernel(const T* __restrict__ src, T* __restrict__ dst, const uint8_t* __restrict__ flags,
+                const LbmParams p) {
+    const size_t plane = (size_t)p.nx * p.ny;
+    const size_t nc = plane * p.nzb;              // SoA stride of one population
+    const size_t c0 = (size_t)p.za * plane;
+    const size_t ncell = (size_t)(p.zb - p.za) * plane;
+    const T omega = T(p.omega);
+    for (size_t t = blockIdx.x * (size_t)blockDim.x + threadIdx.x; t < ncell; t += (size_t)gridDim.x * blockDim.x) {
+        const size_t c = c0 + t;
+        const uint8_t fl = flags[c];
+        T f[19];
+#pragma unroll
+        for (int i = 0; i < 19; ++i) f[i] = src[i * nc + c];
+        if (fl != 0) {
+#pragma unroll
+            for (int i = 0; i < 19; ++i) dst[i * nc + c] = f[i];
+            continue;
+        }
+        collide<T, E>(f, omega);
+        const int nx = p.nx;
+        auto push = [&](auto Ic) {
+            constexpr int I = decltype(Ic)::value;
+            constexpr long long off_c = 0;
+            (void)off_c;
+            const long long off = (long long)D3Q19<I>::ex + (long long)D3Q19<I>::ey * nx +
+                                  (long long)D3Q19<I>::ez * (long long)plane;
+            const size_t tc = (size_t)((long long)c + off);
+            if constexpr (I == 0) {
+                dst[c] = f[0];
+            } else {
+                const uint8_t tf = flags[tc];
+                if (tf == 0) dst[I * nc + tc] = f[I];
+                else if (tf == 1) dst[D3Q19<I>::opp * nc + c] = f[I];
+                else dst[D3Q19<I>::opp * nc + c] = Ar<T, E>::sub(f[I], T(p.lidc[I]));
+            }
+        };
+        [&]<int... Is>(std::integer_sequence<int, Is...>) { (push(std::integral_constant<int, Is>{}), ...); }
+        (std::make_integer_sequence<int, 19>{});
+    }
+}
+
+}  // namespace st35d

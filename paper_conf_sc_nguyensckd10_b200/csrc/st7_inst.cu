@@ -1,0 +1,66 @@
+// st7_inst.cu — instantiates st7_35d_kernel for one (dtype, mode); compiled
+// once per combination with -DST_T=float|double -DST_EXACT=0|1.
+#include "launch.h"
+
+#ifndef ST_T
+#define ST_T float
+#endif
+#ifndef ST_EXACT
+#define ST_EXACT 0
+#endif
+
+#define ST_CAT2(a, b) a##b
+#define ST_CAT(a, b) ST_CAT2(a, b)
+#if ST_EXACT
+#define ST_MODE exact
+#else
+#define ST_MODE fast
+#endif
+// a NAMED per-unit namespace: nvcc emits template instantiations inside an
+// anonymous namespace as weak symbols with identical names in every unit,
+// which the linker would merge across the four (dtype, mode) objects.
+#define ST_UNIT_NS ST_CAT(ST_CAT(ST_CAT(unit_, ST_TNAME), _), ST_MODE)
+
+namespace st35d {
+namespace ST_UNIT_NS {
+
+using TT = ST_T;
+constexpr int NTX = sizeof(TT) == 4 ? 16 : 32;
+
+template <int D, int VY>
+cudaError_t launch(const CUtensorMap* map, const St7Params& p, int grid, int threads, size_t smem,
+                   cudaStream_t s) {
+    auto k = st7_35d_kernel<TT, D, NTX, VY, ST_EXACT != 0, ST7_MAXT>;
+    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    k<<<grid, threads, smem, s>>>(*map, p);
+    return cudaGetLastError();
+}
+
+template <int VY>
+St7LaunchFn pick(int D) {
+    switch (D) {
+        case 1: return launch<1, VY>;
+        case 2: return launch<2, VY>;
+        case 3: return launch<3, VY>;
+        case 4: return launch<4, VY>;
+        case 5: return launch<5, VY>;
+        case 6: return launch<6, VY>;
+        case 7: return launch<7, VY>;
+        case 8: return launch<8, VY>;
+        default: return nullptr;
+    }
+}
+
+}  // namespace ST_UNIT_NS
+using namespace ST_UNIT_NS;
+
+#define ST_FN ST_CAT(ST_CAT(ST_CAT(st7_lookup_, ST_TNAME), _), ST_MODE)
+
+St7LaunchFn ST_FN(int D, int VY) {
+    if (VY == 4) return pick<4>(D);
+    if (VY == 2) return pick<2>(D);
+    return nullptr;
+}
+
+}  // namespace st35d

@@ -1,0 +1,120 @@
+"""GPU parity of the 3.5D 7-point sweep (st7_run through the C ABI) against
+the CPU oracle on the same seeded grids (SURVEY §8(c) gates):
+FP32 max rel err <= 1e-5, FP64 <= 1e-12, bit-exact in the -fmad=false /
+oracle-order build (st_plan_set_bitexact).
+"""
+import numpy as np
+import pytest
+import torch
+
+import stgen
+import paper_conf_sc_nguyensckd10_b200 as st
+
+pytestmark = pytest.mark.gpu
+
+TOL = {np.float32: 1e-5, np.float64: 1e-12}
+
+
+def relerr(g, o):
+    g = g.astype(np.float64)
+    o = o.astype(np.float64)
+    return float(np.max(np.abs(g - o) / np.maximum(np.abs(o), 1e-30)))
+
+
+def run_gpu(a, alpha, beta, T, dim_T, exact=False):
+    nz, ny, nx = a.shape
+    dt = torch.float32 if a.dtype == np.float32 else torch.float64
+    with st.Plan(nx, ny, nz, dt, dim_T) as p:
+        if exact:
+            p.set_bitexact(True)
+        x = torch.from_numpy(a).cuda()
+        y = torch.empty_like(x)
+        p.st7(x, y, alpha, beta, T)
+        p.sync()
+        return y.cpu().numpy(), p.info()
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_config1_64cube(oracle_lib, dtype):
+    # BASELINE configs[0]: 64^3, T=4, dim_T=2, seed 1
+    a = stgen.grid7(64, 64, 64, 1, dtype)
+    ref = oracle_lib.st7(a, 0.4, 0.1, 4)
+    got, _ = run_gpu(a, 0.4, 0.1, 4, 2)
+    assert relerr(got, ref) <= TOL[dtype]
+    got, _ = run_gpu(a, 0.4, 0.1, 4, 2, exact=True)
+    assert np.array_equal(got, ref)
+
+
+SHAPES = [(68, 52, 37), (128, 96, 20), (16, 9, 5), (200, 70, 11)]
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+@pytest.mark.parametrize("dim_T", [1, 2, 3, 4, 5, 6, 7, 8])
+def test_ragged_all_depths(oracle_lib, dtype, dim_T):
+    for k, (nx, ny, nz) in enumerate(SHAPES):
+        if dtype == np.float64 and nx % 2:
+            continue
+        a = stgen.grid7(nx, ny, nz, 100 + k, dtype)
+        T = dim_T * 2 + 1 + k  # several sweeps incl. a remainder sweep
+        ref = oracle_lib.st7(a, 0.4, 0.1, T)
+        got, _ = run_gpu(a, 0.4, 0.1, T, dim_T, exact=True)
+        assert np.array_equal(got, ref), (nx, ny, nz, T)
+        got, _ = run_gpu(a, 0.4, 0.1, T, dim_T)
+        assert relerr(got, ref) <= TOL[dtype] * max(1, T / 10), (nx, ny, nz, T)
+
+
+def test_dimT_invariance_bitexact():
+    a = stgen.grid7(96, 80, 40, 7, np.float32)
+    outs = [run_gpu(a, 0.4, 0.1, 12, d, exact=True)[0] for d in range(1, 9)]
+    for o in outs[1:]:
+        assert np.array_equal(o, outs[0])
+
+
+def test_T0_T1_and_shell(oracle_lib):
+    a = stgen.grid7(64, 40, 30, 3, np.float32)
+    got, _ = run_gpu(a, 0.4, 0.1, 0, 4)
+    assert np.array_equal(got, a)
+    got, _ = run_gpu(a, 0.4, 0.1, 1, 4, exact=True)
+    assert np.array_equal(got, oracle_lib.st7(a, 0.4, 0.1, 1))
+    got, _ = run_gpu(a, 0.4, 0.1, 9, 4)
+    for sl in (np.s_[0], np.s_[-1], np.s_[:, 0], np.s_[:, -1], np.s_[:, :, 0], np.s_[:, :, -1]):
+        assert np.array_equal(got[sl], a[sl])
+
+
+def test_host_pointer_path(oracle_lib):
+    a = stgen.grid7(64, 48, 24, 5, np.float32)
+    out = np.empty_like(a)
+    h = st.st_plan_create(64, 48, 24, st.ST_F32, 3)
+    try:
+        st.st_plan_set_bitexact(h, True)
+        st.st7_run(h, a.copy(), out, 0.4, 0.1, 7)
+    finally:
+        st.st_destroy(h)
+    assert np.array_equal(out, oracle_lib.st7(a, 0.4, 0.1, 7))
+
+
+def test_errors():
+    with pytest.raises(st.StError):
+        st.st_plan_create(2, 64, 64, st.ST_F32, 2)
+    with pytest.raises(st.StError):
+        st.st_plan_create(64, 64, 64, st.ST_F32, 9)
+    with pytest.raises(st.StError):
+        st.st_plan_create(66, 64, 64, st.ST_F32, 2)   # 264 B rows: not a 16 B multiple
+    with st.Plan(64, 64, 64, torch.float32, 2) as p:
+        x = torch.zeros(64, 64, 64, device="cuda")
+        with pytest.raises(st.StError):
+            p.st7(x, x, 0.4, 0.1, 3)                 # aliasing
+        with pytest.raises(st.StError):
+            p.st7(x, torch.empty_like(x), 0.4, 0.1, -1)
+        with pytest.raises(st.StError):
+            p.st7(x, np.empty((64, 64, 64), np.float32), 0.4, 0.1, 1)  # mixed host/device
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_config2_256_sampled(oracle_lib, dtype):
+    # BASELINE configs[1] size in the launch configuration bench.py times (dim_T=4 f32)
+    n, T = 256, 20
+    a = stgen.grid7(n, n, n, 2, dtype)
+    ref = oracle_lib.st7(a, 0.4, 0.1, T)
+    got, info = run_gpu(a, 0.4, 0.1, T, 4 if dtype == np.float32 else 2)
+    assert relerr(got, ref) <= TOL[dtype] * 2
