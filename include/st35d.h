@@ -153,6 +153,7 @@ typedef struct {
     double kappa;           /* eq. (2) analog: computed / useful points         */
     int kernel;             /* internal variant id                               */
     int dim_t_sweep;        /* deepest sweep actually run (<= dim_T, see above)  */
+    int ring;               /* TMA plane-ring slots (ring-2 planes in flight)    */
 } st_plan_info;
 int st_plan_get_info(const st_plan* plan, int lbm, st_plan_info* info);
 

@@ -34,7 +34,8 @@ class st_plan_info(ctypes.Structure):
     _fields_ = [("tile_x", ctypes.c_int), ("tile_y", ctypes.c_int), ("out_x", ctypes.c_int),
                 ("out_y", ctypes.c_int), ("tiles_x", ctypes.c_int), ("tiles_y", ctypes.c_int),
                 ("ctas", ctypes.c_int), ("threads", ctypes.c_int), ("smem_bytes", ctypes.c_int),
-                ("kappa", ctypes.c_double), ("kernel", ctypes.c_int), ("dim_t_sweep", ctypes.c_int)]
+                ("kappa", ctypes.c_double), ("kernel", ctypes.c_int), ("dim_t_sweep", ctypes.c_int),
+                ("ring", ctypes.c_int)]
 
 
 class st_blocking(ctypes.Structure):

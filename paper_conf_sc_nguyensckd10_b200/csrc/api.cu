@@ -76,7 +76,7 @@ static int encode_3d(CUtensorMap* map, const void* base, st_dtype dt, int nx, in
 // ----------------------------------------------------------------------------
 struct Geo7 {
     int d = 0, VY = 0, NTX = 0, VX = 0, TX = 0, NTY = 0, TY = 0;
-    int hx = 0, wx = 0, wy = 0, tiles_x = 0, tiles_y = 0, threads = 0, grid = 0;
+    int hx = 0, wx = 0, wy = 0, tiles_x = 0, tiles_y = 0, threads = 0, grid = 0, maxt = 0, ring = 4;
     size_t smem = 0;
     double kappa = 0;
     St7LaunchFn fn = nullptr;
@@ -109,20 +109,28 @@ struct st_plan {
 
 static size_t esize(st_dtype d) { return d == ST_F32 ? 4 : 8; }
 
-static int vy_for(st_dtype dt, int d) {
-    // register budget of the (D, VY) instantiations (ptxas -v: no spills)
-    if (dt == ST_F32) return d <= 4 ? 4 : 2;
-    return d <= 2 ? 4 : 2;
+// Kernel variant (rows per thread VY, max threads per CTA) for a sweep depth:
+// the register budget of each (D, VY, MAXT) instantiation, from ptxas -v
+// (no spills): 512 threads cap registers at 128 and double the resident
+// warps; 256 threads allow 255 registers for the deeper Z windows.
+static void variant_for(st_dtype dt, int d, int& vy, int& maxt) {
+    if (const char* e = getenv("ST_VARIANT")) {  // "VYxMAXT", e.g. 4x256 (tuning only)
+        int a = 0, b = 0;
+        if (sscanf(e, "%dx%d", &a, &b) == 2) { vy = a; maxt = b; return; }
+    }
+    if (dt == ST_F32) { vy = d <= 4 ? 2 : 2; maxt = d <= 4 ? 512 : 256; return; }
+    vy = 2; maxt = d <= 3 ? 512 : 256;
 }
 
-static St7LaunchFn lookup7(st_dtype dt, bool exact, int d, int vy) {
-    if (dt == ST_F32) return exact ? st7_lookup_f32_exact(d, vy) : st7_lookup_f32_fast(d, vy);
-    return exact ? st7_lookup_f64_exact(d, vy) : st7_lookup_f64_fast(d, vy);
+static St7LaunchFn lookup7(st_dtype dt, bool exact, int d, int vy, int maxt) {
+    if (dt == ST_F32) return exact ? st7_lookup_f32_exact(d, vy, maxt) : st7_lookup_f32_fast(d, vy, maxt);
+    return exact ? st7_lookup_f64_exact(d, vy, maxt) : st7_lookup_f64_fast(d, vy, maxt);
 }
 
-static size_t smem7(const Geo7& g, st_dtype dt) {
-    return (size_t)ST7_RING * g.TX * g.TY * esize(dt) + (size_t)(g.d > 1 ? g.d - 1 : 0) * 4 * g.threads * 16 +
-           ST7_RING * 8;
+static size_t smem7(const Geo7& g, st_dtype dt, int ring) {
+    // TMA ring + row exchange [D-1][2][2][MAXT] x 16 B + mbarriers
+    return (size_t)ring * g.TX * g.TY * esize(dt) + (size_t)(g.d > 1 ? g.d - 1 : 0) * 4 * g.maxt * 16 +
+           ring * 8;
 }
 
 // Planner for one sweep depth d over an nx x ny plane with nzo output planes:
@@ -135,12 +143,12 @@ static int plan7(st_plan* p, int d, int nzo, Geo7& g) {
     g.VX = p->dtype == ST_F32 ? 4 : 2;
     g.NTX = p->dtype == ST_F32 ? 16 : 32;
     g.TX = g.NTX * g.VX;
-    g.VY = vy_for(p->dtype, d);
+    variant_for(p->dtype, d, g.VY, g.maxt);
     g.hx = (d + g.VX - 1) / g.VX * g.VX;
     g.wx = (g.TX - g.hx - d) & ~(g.VX - 1);
     if (g.wx < g.VX) return fail(ST_EUNSUPPORTED, "dim_T %d too deep for a %d-wide tile", d, g.TX);
     g.tiles_x = (p->nx + g.wx - 1) / g.wx;
-    const int ntymax = ST7_MAXT / g.NTX;
+    const int ntymax = g.maxt / g.NTX;
     long best = -1;
     for (int nty = 2; nty <= ntymax; ++nty) {
         Geo7 c = g;
@@ -150,8 +158,14 @@ static int plan7(st_plan* p, int d, int nzo, Geo7& g) {
         c.wy = c.TY - 2 * d;
         if (c.wy < 1) continue;
         c.tiles_y = (p->ny + c.wy - 1) / c.wy;
-        c.smem = smem7(c, p->dtype);
-        if (c.smem > p->smem_optin) continue;
+        // TMA ring: as deep as shared memory allows (prefetch ring-2 planes ahead:
+        // the plane loads must cover HBM latency, several rounds of compute)
+        c.ring = 0;
+        for (int r = ST7_RING_MAX; r >= 4; --r)
+            if (smem7(c, p->dtype, r) <= p->smem_optin) { c.ring = r; break; }
+        if (const char* e = getenv("ST_RING")) c.ring = std::min(c.ring, atoi(e));
+        if (c.ring < 4) continue;
+        c.smem = smem7(c, p->dtype, c.ring);
         long cost = (long)c.tiles_y * c.TY;
         if (best < 0 || cost < best || (cost == best && c.TY > g.TY)) {
             best = cost;
@@ -162,14 +176,14 @@ static int plan7(st_plan* p, int d, int nzo, Geo7& g) {
     const long long work = (long long)g.tiles_x * g.tiles_y * nzo;
     g.grid = (int)std::min<long long>(p->sms, std::max<long long>(work, 1));
     g.kappa = (double)g.tiles_x * g.TX * g.tiles_y * g.TY / ((double)p->nx * p->ny);
-    g.fn = lookup7(p->dtype, p->exact, d, g.VY);
+    g.fn = lookup7(p->dtype, p->exact, d, g.VY, g.maxt);
     if (!g.fn) return fail(ST_EUNSUPPORTED, "no kernel for dim_T %d", d);
     return ST_OK;
 }
 
 static int get_geo7(st_plan* p, int d, int nzo, Geo7*& out) {
     auto it = p->geo7.find(d);
-    if (it == p->geo7.end() || it->second.fn != lookup7(p->dtype, p->exact, d, it->second.VY)) {
+    if (it == p->geo7.end() || it->second.fn != lookup7(p->dtype, p->exact, d, it->second.VY, it->second.maxt)) {
         Geo7 g;
         int rc = plan7(p, d, nzo, g);
         if (rc) return rc;
@@ -286,8 +300,9 @@ extern "C" int st_plan_get_info(const st_plan* p, int lbm, st_plan_info* info) {
     const Geo7& g = it->second;
     info->tile_x = g.TX; info->tile_y = g.TY; info->out_x = g.wx; info->out_y = g.wy;
     info->tiles_x = g.tiles_x; info->tiles_y = g.tiles_y; info->ctas = g.grid; info->threads = g.threads;
-    info->smem_bytes = (int)g.smem; info->kappa = g.kappa; info->kernel = g.VY;
+    info->smem_bytes = (int)g.smem; info->kappa = g.kappa; info->kernel = g.VY * 1000 + g.maxt;
     info->dim_t_sweep = p->dimK;
+    info->ring = g.ring;
     return ST_OK;
 }
 
@@ -344,6 +359,8 @@ static int launch7(st_plan* p, const void* src, void* dst, int d, double alpha, 
     prm.tiles_x = g->tiles_x; prm.ntiles = g->tiles_x * g->tiles_y;
     prm.wx = g->wx; prm.wy = g->wy; prm.hx = g->hx;
     prm.work = (long long)prm.ntiles * (sv.zb - sv.za);
+    prm.ring = g->ring;
+    if (const char* e = getenv("ST_DBG")) prm.dbg = atoi(e);
     prm.alpha = alpha; prm.beta = beta;
     if (prm.work <= 0) return ST_OK;
     cudaError_t e = g->fn(&map, prm, g->grid, g->threads, g->smem, sv.stream ? sv.stream : p->stream);

@@ -12,10 +12,10 @@ using St7LaunchFn = cudaError_t (*)(const CUtensorMap* map, const St7Params& p, 
                                     size_t smem, cudaStream_t s);
 
 // returns nullptr if (D, VY) is not compiled
-St7LaunchFn st7_lookup_f32_fast(int D, int VY);
-St7LaunchFn st7_lookup_f32_exact(int D, int VY);
-St7LaunchFn st7_lookup_f64_fast(int D, int VY);
-St7LaunchFn st7_lookup_f64_exact(int D, int VY);
+St7LaunchFn st7_lookup_f32_fast(int D, int VY, int MAXT);
+St7LaunchFn st7_lookup_f32_exact(int D, int VY, int MAXT);
+St7LaunchFn st7_lookup_f64_fast(int D, int VY, int MAXT);
+St7LaunchFn st7_lookup_f64_exact(int D, int VY, int MAXT);
 
 cudaError_t lbm_push_launch(int dtype, bool exact, const void* src, void* dst, const uint8_t* flags,
                             const LbmParams& p, int grid, cudaStream_t s);

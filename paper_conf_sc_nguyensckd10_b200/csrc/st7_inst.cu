@@ -27,27 +27,27 @@ namespace ST_UNIT_NS {
 using TT = ST_T;
 constexpr int NTX = sizeof(TT) == 4 ? 16 : 32;
 
-template <int D, int VY>
+template <int D, int VY, int MAXT>
 cudaError_t launch(const CUtensorMap* map, const St7Params& p, int grid, int threads, size_t smem,
                    cudaStream_t s) {
-    auto k = st7_35d_kernel<TT, D, NTX, VY, ST_EXACT != 0, ST7_MAXT>;
+    auto k = st7_35d_kernel<TT, D, NTX, VY, ST_EXACT != 0, MAXT>;
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     k<<<grid, threads, smem, s>>>(*map, p);
     return cudaGetLastError();
 }
 
-template <int VY>
+template <int VY, int MAXT>
 St7LaunchFn pick(int D) {
     switch (D) {
-        case 1: return launch<1, VY>;
-        case 2: return launch<2, VY>;
-        case 3: return launch<3, VY>;
-        case 4: return launch<4, VY>;
-        case 5: return launch<5, VY>;
-        case 6: return launch<6, VY>;
-        case 7: return launch<7, VY>;
-        case 8: return launch<8, VY>;
+        case 1: return launch<1, VY, MAXT>;
+        case 2: return launch<2, VY, MAXT>;
+        case 3: return launch<3, VY, MAXT>;
+        case 4: return launch<4, VY, MAXT>;
+        case 5: return launch<5, VY, MAXT>;
+        case 6: return launch<6, VY, MAXT>;
+        case 7: return launch<7, VY, MAXT>;
+        case 8: return launch<8, VY, MAXT>;
         default: return nullptr;
     }
 }
@@ -57,9 +57,11 @@ using namespace ST_UNIT_NS;
 
 #define ST_FN ST_CAT(ST_CAT(ST_CAT(st7_lookup_, ST_TNAME), _), ST_MODE)
 
-St7LaunchFn ST_FN(int D, int VY) {
-    if (VY == 4) return pick<4>(D);
-    if (VY == 2) return pick<2>(D);
+// variants: (VY=4, 256 threads max), (VY=2, 256), (VY=2, 512 threads: <= 128 registers)
+St7LaunchFn ST_FN(int D, int VY, int MAXT) {
+    if (VY == 4 && MAXT == 256) return pick<4, 256>(D);
+    if (VY == 2 && MAXT == 256) return pick<2, 256>(D);
+    if (VY == 2 && MAXT == 512) return pick<2, 512>(D);
     return nullptr;
 }
 

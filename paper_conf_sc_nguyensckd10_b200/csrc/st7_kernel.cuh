@@ -41,142 +41,206 @@ struct St7Params {
     int wx, wy;        // written region per tile
     int hx;            // x halo (>= D, multiple of VX)
     long long work;    // ntiles * (zb - za)
+    int ring;          // TMA ring slots (<= ST7_RING_MAX); ring - 2 planes are prefetched ahead
+    int dbg;           // tuning only: bit 0 = stream planes without computing levels
     double alpha, beta;
 };
 
-constexpr int ST7_RING = 4;   // TMA ring slots
-constexpr int ST7_PF = 2;     // planes prefetched ahead
+constexpr int ST7_RING_MAX = 12;
 
-template <typename T>
-__device__ __forceinline__ T st7_point(T c, T xm, T xp, T ym, T yp, T zm, T zp, T al, T be, bool exact) {
-    if (exact) {
-        // oracle order (X2): ((x- + x+) + (y- + y+)) + (z- + z+); two products, one add
-        T sx = __dadd_rn(xm, xp), sy = __dadd_rn(ym, yp), sz = __dadd_rn(zm, zp);
-        T s = __dadd_rn(__dadd_rn(sx, sy), sz);
-        return __dadd_rn(__dmul_rn(al, c), __dmul_rn(be, s));
-    } else {
-        T s = ((xm + xp) + (ym + yp)) + (zm + zp);
-        return fma(al, c, be * s);
+// ---------------------------------------------------------------------------
+// One thread's register block of one plane: VY rows x VX columns.
+//  * FP32 (VX = 4): each row is held as two packed pairs a = (c0, c2),
+//    b = (c1, c3) so the X neighbours of one pair are the other pair (plus one
+//    shuffled edge value), and every 7-point update of a pair is 7 packed
+//    sm_100a instructions (FADD2 x5, FMUL2, FFMA2) for 2 points.
+//  * FP64 (VX = 2): plain scalars (the DP pipe is half rate; no packed form).
+// The arithmetic order is the oracle's (X2): ((x- + x+) + (y- + y+)) + (z- + z+),
+// then alpha*c + beta*s; the _rn intrinsics are never contracted, so the
+// bit-exact build only differs by using FMUL2 + FADD2 instead of FFMA2.
+// ---------------------------------------------------------------------------
+template <typename T, int VY> struct Blk;
+template <typename T> struct Row;
+
+template <> struct Row<float> { float2 a, b; };
+template <> struct Row<double> { double v[2]; };
+
+template <int VY> struct Blk<float, VY> {
+    float2 a[VY], b[VY];
+    __device__ __forceinline__ void load_nat(int j, const float* s) {   // smem, natural order
+        const float4 v = *reinterpret_cast<const float4*>(s);
+        a[j] = make_float2(v.x, v.z);
+        b[j] = make_float2(v.y, v.w);
     }
-}
-template <>
-__device__ __forceinline__ float st7_point<float>(float c, float xm, float xp, float ym, float yp, float zm,
-                                                  float zp, float al, float be, bool exact) {
-    if (exact) {
-        float sx = __fadd_rn(xm, xp), sy = __fadd_rn(ym, yp), sz = __fadd_rn(zm, zp);
-        float s = __fadd_rn(__fadd_rn(sx, sy), sz);
-        return __fadd_rn(__fmul_rn(al, c), __fmul_rn(be, s));
-    } else {
-        float s = ((xm + xp) + (ym + yp)) + (zm + zp);
-        return fmaf(al, c, be * s);
+    __device__ __forceinline__ void store_x(int j, float4* s) const {   // exchange row, pair order
+        *s = make_float4(a[j].x, a[j].y, b[j].x, b[j].y);
     }
-}
-
-template <typename T, int VX>
-__device__ __forceinline__ void vload(T (&dst)[VX], const T* src) {
-    using V = typename Vec<T>::type;
-    V v = *reinterpret_cast<const V*>(src);
-    if constexpr (VX == 4) { dst[0] = v.x; dst[1] = v.y; dst[2] = v.z; dst[3] = v.w; }
-    else { dst[0] = v.x; dst[1] = v.y; }
-}
-template <typename T, int VX>
-__device__ __forceinline__ void vstore(T* dst, const T (&s)[VX]) {
-    using V = typename Vec<T>::type;
-    if constexpr (VX == 4) *reinterpret_cast<V*>(dst) = V{s[0], s[1], s[2], s[3]};
-    else *reinterpret_cast<V*>(dst) = V{s[0], s[1]};
-}
-template <typename T, int VX>
-__device__ __forceinline__ void gstore(T* dst, const T (&s)[VX]) {
-    if constexpr (VX == 4) st_global_v4(reinterpret_cast<float*>(dst), make_float4(s[0], s[1], s[2], s[3]));
-    else st_global_v2(reinterpret_cast<double*>(dst), make_double2(s[0], s[1]));
-}
-
-template <typename T, int D, int NTX, int VY, bool EXACT>
-struct St7Sweep {
-    static constexpr int VX = Vec<T>::N;
-    static constexpr int TX = NTX * VX;
-
-    // per-thread register planes: level l (0..D-1), rotating slot k (0..2)
-    T pl[D][3][VY][VX];
-    T outv[VY][VX];
-
-    // block geometry
-    int tx, ty, NTY, TY;
-    // segment geometry
-    int Lx, Ly, ox0, ox1, oy0, oy1;
-    uint32_t fixmask;      // bit j*VX+i: point is on the grid shell or outside (copied)
-    bool wfix;             // warp-uniform: some lane of the warp has fixmask != 0
-    T al, be;
-
-    __device__ __forceinline__ void compute_level(const T (&ZM)[VY][VX], const T (&C)[VY][VX],
-                                                  const T (&ZP)[VY][VX], const T* top, const T* bot,
-                                                  bool zfix, T (&R)[VY][VX]) {
-        T up[VX], dn[VX];
-#pragma unroll
-        for (int i = 0; i < VX; ++i) { up[i] = top[i]; dn[i] = bot[i]; }
-        T left[VY], right[VY];
-#pragma unroll
-        for (int j = 0; j < VY; ++j) {
-            left[j] = __shfl_up_sync(0xffffffffu, C[j][VX - 1], 1, NTX);
-            right[j] = __shfl_down_sync(0xffffffffu, C[j][0], 1, NTX);
-        }
-        if (zfix) {
-#pragma unroll
-            for (int j = 0; j < VY; ++j)
-#pragma unroll
-                for (int i = 0; i < VX; ++i) R[j][i] = C[j][i];
-            return;
-        }
-#pragma unroll
-        for (int j = 0; j < VY; ++j)
-#pragma unroll
-            for (int i = 0; i < VX; ++i) {
-                T xm = i > 0 ? C[j][i - 1] : left[j];
-                T xp = i < VX - 1 ? C[j][i + 1] : right[j];
-                T ym = j > 0 ? C[j - 1][i] : up[i];
-                T yp = j < VY - 1 ? C[j + 1][i] : dn[i];
-                R[j][i] = st7_point<T>(C[j][i], xm, xp, ym, yp, ZM[j][i], ZP[j][i], al, be, EXACT);
-            }
-        if (wfix) {  // warp-uniform: only warps touching the grid shell pay for the selects
-#pragma unroll
-            for (int j = 0; j < VY; ++j)
-#pragma unroll
-                for (int i = 0; i < VX; ++i)
-                    if (fixmask & (1u << (j * VX + i))) R[j][i] = C[j][i];
-        }
+    __device__ __forceinline__ void store_global(int j, float* g) const {
+        st_global_v4(g, make_float4(a[j].x, b[j].x, a[j].y, b[j].y));
     }
 };
+template <int VY> struct Blk<double, VY> {
+    double v[VY][2];
+    __device__ __forceinline__ void load_nat(int j, const double* s) {
+        const double2 t = *reinterpret_cast<const double2*>(s);
+        v[j][0] = t.x; v[j][1] = t.y;
+    }
+    __device__ __forceinline__ void store_x(int j, double2* s) const { *s = make_double2(v[j][0], v[j][1]); }
+    __device__ __forceinline__ void store_global(int j, double* g) const {
+        st_global_v2(g, make_double2(v[j][0], v[j][1]));
+    }
+};
+
+__device__ __forceinline__ Row<float> row_nat(const float* s) {
+    const float4 v = *reinterpret_cast<const float4*>(s);
+    return Row<float>{make_float2(v.x, v.z), make_float2(v.y, v.w)};
+}
+__device__ __forceinline__ Row<float> row_x(const float4* s) {
+    const float4 v = *s;
+    return Row<float>{make_float2(v.x, v.y), make_float2(v.z, v.w)};
+}
+__device__ __forceinline__ Row<double> row_nat(const double* s) {
+    const double2 v = *reinterpret_cast<const double2*>(s);
+    return Row<double>{{v.x, v.y}};
+}
+__device__ __forceinline__ Row<double> row_x(const double2* s) {
+    const double2 v = *s;
+    return Row<double>{{v.x, v.y}};
+}
+
+// Bit-exact combine alpha*c + beta*s: ptxas 12.9 fuses mul.rn.f32x2 followed by
+// add.rn.f32x2 into FFMA2 even with -fmad=false, so the exact build does the
+// final combine with scalar __fmul_rn / __fadd_rn (which are never fused).
+__device__ __forceinline__ float2 combine_exact(float al, float2 c, float be, float2 s) {
+    return make_float2(__fadd_rn(__fmul_rn(al, c.x), __fmul_rn(be, s.x)),
+                       __fadd_rn(__fmul_rn(al, c.y), __fmul_rn(be, s.y)));
+}
+
+// Per-thread update coefficients.  A point on the x shell (x = 0 or nx-1)
+// is Dirichlet-fixed: it gets alpha = 1, beta = 0, so alpha*c + beta*s == c
+// exactly (s is always finite here: every neighbour is loaded data or a
+// finite combination of it).  Rows on the y shell are copied in a rare
+// warp-uniform branch; whole z-shell planes use Coef::fixed().
+template <typename T> struct Coef;
+template <> struct Coef<float> {
+    float2 alA, beA, alB, beB;     // for the pairs a = (c0, c2), b = (c1, c3)
+    static __device__ __forceinline__ Coef fixed() {
+        return Coef{make_float2(1.f, 1.f), make_float2(0.f, 0.f), make_float2(1.f, 1.f), make_float2(0.f, 0.f)};
+    }
+    static __device__ __forceinline__ Coef make(float al, float be, uint32_t xfix) {  // xfix bit i: column i fixed
+        Coef k;
+        k.alA = make_float2(xfix & 1 ? 1.f : al, xfix & 4 ? 1.f : al);
+        k.beA = make_float2(xfix & 1 ? 0.f : be, xfix & 4 ? 0.f : be);
+        k.alB = make_float2(xfix & 2 ? 1.f : al, xfix & 8 ? 1.f : al);
+        k.beB = make_float2(xfix & 2 ? 0.f : be, xfix & 8 ? 0.f : be);
+        return k;
+    }
+};
+template <> struct Coef<double> {
+    double al[2], be[2];
+    static __device__ __forceinline__ Coef fixed() { return Coef{{1.0, 1.0}, {0.0, 0.0}}; }
+    static __device__ __forceinline__ Coef make(double al, double be, uint32_t xfix) {
+        return Coef{{xfix & 1 ? 1.0 : al, xfix & 2 ? 1.0 : al}, {xfix & 1 ? 0.0 : be, xfix & 2 ? 0.0 : be}};
+    }
+};
+
+// one level of the sweep for one thread's block: R = stencil(ZM, C, ZP)
+template <int NTX, int VY, bool EXACT>
+__device__ __forceinline__ void st7_level(const Blk<float, VY>& ZM, const Blk<float, VY>& C,
+                                          const Blk<float, VY>& ZP, const Row<float>& top,
+                                          const Row<float>& bot, const Coef<float>& k, bool yslow,
+                                          uint32_t rowfix, Blk<float, VY>& R) {
+#pragma unroll
+    for (int j = 0; j < VY; ++j) {
+        const float left = __shfl_up_sync(0xffffffffu, C.b[j].y, 1, NTX);     // x0 - 1
+        const float right = __shfl_down_sync(0xffffffffu, C.a[j].x, 1, NTX);  // x0 + 4
+        const float2 yma = j > 0 ? C.a[j - 1] : top.a, ypa = j < VY - 1 ? C.a[j + 1] : bot.a;
+        const float2 ymb = j > 0 ? C.b[j - 1] : top.b, ypb = j < VY - 1 ? C.b[j + 1] : bot.b;
+        const float2 sxa = __fadd2_rn(make_float2(left, C.b[j].x), C.b[j]);
+        const float2 sxb = __fadd2_rn(C.a[j], make_float2(C.a[j].y, right));
+        const float2 sa = __fadd2_rn(__fadd2_rn(sxa, __fadd2_rn(yma, ypa)), __fadd2_rn(ZM.a[j], ZP.a[j]));
+        const float2 sb = __fadd2_rn(__fadd2_rn(sxb, __fadd2_rn(ymb, ypb)), __fadd2_rn(ZM.b[j], ZP.b[j]));
+        if (EXACT) {
+            R.a[j] = make_float2(__fadd_rn(__fmul_rn(k.alA.x, C.a[j].x), __fmul_rn(k.beA.x, sa.x)),
+                                 __fadd_rn(__fmul_rn(k.alA.y, C.a[j].y), __fmul_rn(k.beA.y, sa.y)));
+            R.b[j] = make_float2(__fadd_rn(__fmul_rn(k.alB.x, C.b[j].x), __fmul_rn(k.beB.x, sb.x)),
+                                 __fadd_rn(__fmul_rn(k.alB.y, C.b[j].y), __fmul_rn(k.beB.y, sb.y)));
+        } else {
+            R.a[j] = __ffma2_rn(k.alA, C.a[j], __fmul2_rn(k.beA, sa));
+            R.b[j] = __ffma2_rn(k.alB, C.b[j], __fmul2_rn(k.beB, sb));
+        }
+    }
+    if (yslow) {  // warp-uniform: only warps holding a y-shell row
+#pragma unroll
+        for (int j = 0; j < VY; ++j)
+            if (rowfix & (1u << j)) { R.a[j] = C.a[j]; R.b[j] = C.b[j]; }
+    }
+}
+
+template <int NTX, int VY, bool EXACT>
+__device__ __forceinline__ void st7_level(const Blk<double, VY>& ZM, const Blk<double, VY>& C,
+                                          const Blk<double, VY>& ZP, const Row<double>& top,
+                                          const Row<double>& bot, const Coef<double>& k, bool yslow,
+                                          uint32_t rowfix, Blk<double, VY>& R) {
+#pragma unroll
+    for (int j = 0; j < VY; ++j) {
+        const double left = __shfl_up_sync(0xffffffffu, C.v[j][1], 1, NTX);
+        const double right = __shfl_down_sync(0xffffffffu, C.v[j][0], 1, NTX);
+#pragma unroll
+        for (int i = 0; i < 2; ++i) {
+            const double c = C.v[j][i];
+            const double xm = i == 0 ? left : C.v[j][0], xp = i == 1 ? right : C.v[j][1];
+            const double ym = j > 0 ? C.v[j - 1][i] : top.v[i], yp = j < VY - 1 ? C.v[j + 1][i] : bot.v[i];
+            const double sx = __dadd_rn(xm, xp), sy = __dadd_rn(ym, yp), sz = __dadd_rn(ZM.v[j][i], ZP.v[j][i]);
+            const double s = __dadd_rn(__dadd_rn(sx, sy), sz);
+            R.v[j][i] = EXACT ? __dadd_rn(__dmul_rn(k.al[i], c), __dmul_rn(k.be[i], s))
+                              : __fma_rn(k.al[i], c, __dmul_rn(k.be[i], s));
+        }
+    }
+    if (yslow) {
+#pragma unroll
+        for (int j = 0; j < VY; ++j)
+            if (rowfix & (1u << j)) { R.v[j][0] = C.v[j][0]; R.v[j][1] = C.v[j][1]; }
+    }
+}
 
 template <typename T, int D, int NTX, int VY, bool EXACT, int MAXT>
 __global__ void __launch_bounds__(MAXT, 1)
 st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
-    using S = St7Sweep<T, D, NTX, VY, EXACT>;
-    constexpr int VX = S::VX;
-    constexpr int TX = S::TX;
+    constexpr int VX = Vec<T>::N;
+    constexpr int TX = NTX * VX;
     using V = typename Vec<T>::type;
+    using B = Blk<T, VY>;
 
     extern __shared__ __align__(128) unsigned char smem_raw[];
-    S st;
-    st.tx = threadIdx.x % NTX;
-    st.ty = threadIdx.x / NTX;
-    st.NTY = blockDim.x / NTX;
-    st.TY = st.NTY * VY;
-    const int NT = blockDim.x;
-    const int TY = st.TY;
-    st.al = T(p.alpha);
-    st.be = T(p.beta);
+    const int tid = threadIdx.x;
+    const int tx = tid % NTX;
+    const int ty = tid / NTX;
+    const int NTY = blockDim.x / NTX;
+    const int TY = NTY * VY;
+    const T al = T(p.alpha), be = T(p.beta);
 
-    T* ring = reinterpret_cast<T*>(smem_raw);                      // [ST7_RING][TY][TX]
+    const int RING = p.ring, PF = p.ring - 2;
+    T* ring = reinterpret_cast<T*>(smem_raw);                      // [RING][TY][TX]
     const int slot_elems = TX * TY;
-    V* xbuf = reinterpret_cast<V*>(ring + ST7_RING * slot_elems);  // [D-1][2 parity][2 N/S][NT]
-    uint64_t* bars = reinterpret_cast<uint64_t*>(xbuf + (D > 1 ? (D - 1) * 4 * NT : 0));
+    // row exchange buffer [level 1..D-1][parity][N row / S row][MAXT] (16-byte rows)
+    V* xbuf = reinterpret_cast<V*>(ring + RING * slot_elems);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(xbuf + (D > 1 ? (D - 1) * 4 * MAXT : 0));
 
-    if (threadIdx.x == 0) {
+    if (tid == 0) {
         prefetch_tensormap(&tmap);
-        for (int s = 0; s < ST7_RING; ++s) mbar_init(&bars[s], 1);
+        for (int s = 0; s < RING; ++s) mbar_init(&bars[s], 1);
         fence_mbar_init();
     }
     __syncthreads();
+
+    // register planes: level l (0..D-1), rotating slot (prev / cur / new)
+    B pl[D][3];
+    B outv;
+#pragma unroll
+    for (int l = 0; l < D; ++l)
+#pragma unroll
+        for (int k = 0; k < 3; ++k) pl[l][k] = B{};   // finite (see Coef)
 
     const int nzo = p.zb - p.za;
     const long long G = gridDim.x;
@@ -187,10 +251,13 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
     const uint32_t tile_bytes = (uint32_t)(slot_elems * sizeof(T));
     uint32_t nload = 0;       // loads issued by this CTA so far (ring index)
 
-    const int tyu = max(st.ty - 1, 0), tyd = min(st.ty + 1, st.NTY - 1);
-    const int my_off = (VY * st.ty) * TX + VX * st.tx;                 // my first row in a plane
-    const int top_off = max(VY * st.ty - 1, 0) * TX + VX * st.tx;       // row above my block
-    const int bot_off = min(VY * st.ty + VY, TY - 1) * TX + VX * st.tx; // row below my block
+    const int tyu = max(ty - 1, 0), tyd = min(ty + 1, NTY - 1);
+    const int my_off = (VY * ty) * TX + VX * tx;                   // my first row in a plane
+    const int top_off = max(VY * ty - 1, 0) * TX + VX * tx;         // row above my block
+    const int bot_off = min(VY * ty + VY, TY - 1) * TX + VX * tx;   // row below my block
+    V* const xw = xbuf + tid;                                      // my N row (S row at + MAXT)
+    const V* const xtop = xbuf + MAXT + tyu * NTX + tx;            // S row of the block above
+    const V* const xbot = xbuf + tyd * NTX + tx;                   // N row of the block below
     T* outp = reinterpret_cast<T*>(p.out);
     const size_t plane = (size_t)p.nx * p.ny;
 
@@ -203,104 +270,124 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
         item = seg_end;
 
         const int ix = tile % p.tiles_x, iy = tile / p.tiles_x;
-        st.ox0 = ix * p.wx; st.ox1 = min(st.ox0 + p.wx, p.nx);
-        st.oy0 = iy * p.wy; st.oy1 = min(st.oy0 + p.wy, p.ny);
-        st.Lx = st.ox0 - p.hx;
-        st.Ly = st.oy0 - D;
-        st.fixmask = 0;
+        const int ox0 = ix * p.wx, ox1 = min(ox0 + p.wx, p.nx);
+        const int oy0 = iy * p.wy, oy1 = min(oy0 + p.wy, p.ny);
+        const int Lx = ox0 - p.hx;
+        const int Ly = oy0 - D;
+        const int xg0 = Lx + VX * tx;
+        uint32_t xfix = 0, rowfix = 0, rowmask = 0;
 #pragma unroll
-        for (int j = 0; j < VY; ++j)
+        for (int i = 0; i < VX; ++i)
+            if (xg0 + i == 0 || xg0 + i == p.nx - 1) xfix |= 1u << i;
 #pragma unroll
-            for (int i = 0; i < VX; ++i) {
-                int xg = st.Lx + VX * st.tx + i, yg = st.Ly + VY * st.ty + j;
-                bool interior = xg >= 1 && xg <= p.nx - 2 && yg >= 1 && yg <= p.ny - 2;
-                if (!interior) st.fixmask |= 1u << (j * VX + i);
-            }
-        st.wfix = __any_sync(0xffffffffu, st.fixmask != 0);
+        for (int j = 0; j < VY; ++j) {
+            const int yg = Ly + VY * ty + j;
+            if (yg >= oy0 && yg < oy1) rowmask |= 1u << j;
+            if (yg == 0 || yg == p.ny - 1) rowfix |= 1u << j;
+        }
+        const bool yslow = __any_sync(0xffffffffu, rowfix != 0);
+        if (!(xg0 >= ox0 && xg0 < ox1)) rowmask = 0;    // quads are all-in or all-out in x
+        const Coef<T> kc = Coef<T>::make(al, be, xfix);
+        T* const outcol = outp + xg0 + (size_t)(Ly + VY * ty) * p.nx;
 
-        // level-0 planes to load, and rounds
+        // level-0 planes to load, rounds, and the steady rounds (every level
+        // active, no z-shell plane): those run without any per-level check
         const int rl0 = max(za - D, zmin);
         const int rl1 = min(zb - 1 + D, zmax);
         const int r0 = rl0;
         const int r1 = zb - 1 + D;
+        const int rs0 = max(max(za + D, zmin + D), -p.zbase + D + 1);
+        const int rs1 = min(min(zb - 1 + D, zmax + 1), min(rl1, p.nzg - 1 - p.zbase));
         const uint32_t kbase = nload;
-        if (threadIdx.x == 0) {
-            for (int q = rl0; q <= min(rl0 + ST7_PF - 1, rl1); ++q) {
-                uint32_t k = kbase + (q - rl0);
-                uint64_t* bar = &bars[k % ST7_RING];
+        if (tid == 0) {
+            for (int q = rl0; q <= min(rl0 + PF - 1, rl1); ++q) {
+                const uint32_t k = kbase + (q - rl0);
+                uint64_t* bar = &bars[k % RING];
                 mbar_arrive_expect_tx(bar, tile_bytes);
-                tma_load_3d(ring + (k % ST7_RING) * slot_elems, &tmap, bar, st.Lx, st.Ly, q);
+                tma_load_3d(ring + (k % RING) * slot_elems, &tmap, bar, Lx, Ly, q);
             }
         }
         nload = kbase + (uint32_t)max(0, rl1 - rl0 + 1);
+        // ring slot / parity of plane q, tracked incrementally (no division in the loop)
+        uint32_t slot_r = kbase % RING, par_r = (kbase / RING) & 1;       // for plane r
+        uint32_t slot_f = (kbase + PF) % RING;                            // for plane r + PF
+        uint32_t slot_m1 = (slot_r + RING - 1) % RING;                    // for plane r - 1
 
-        auto round = [&](auto PHc, int r) {
+        auto round = [&](auto PHc, auto STEADYc, int r) {
             constexpr int PH = decltype(PHc)::value;
+            constexpr bool STEADY = decltype(STEADYc)::value;
             constexpr int PREV = PH % 3, CUR = (PH + 1) % 3, NEW = (PH + 2) % 3;
-            // issue the load of plane r + PF (slot freed by the barrier that ended round r-1)
-            if (threadIdx.x == 0 && r + ST7_PF <= rl1) {
-                uint32_t k = kbase + (r + ST7_PF - rl0);
-                uint64_t* bar = &bars[k % ST7_RING];
+            // issue the load of plane r + PF (its slot was freed by the barrier that ended round r-1)
+            if (tid == 0 && r + PF <= rl1) {
+                uint64_t* bar = &bars[slot_f];
                 mbar_arrive_expect_tx(bar, tile_bytes);
-                tma_load_3d(ring + (k % ST7_RING) * slot_elems, &tmap, bar, st.Lx, st.Ly, r + ST7_PF);
+                tma_load_3d(ring + slot_f * slot_elems, &tmap, bar, Lx, Ly, r + PF);
             }
             // level 0: plane r from the ring into registers
-            if (r <= rl1) {
-                uint32_t k = kbase + (r - rl0);
-                mbar_wait(&bars[k % ST7_RING], (k / ST7_RING) & 1);
-                const T* sl = ring + (k % ST7_RING) * slot_elems;
+            if (STEADY || r <= rl1) {
+                mbar_wait(&bars[slot_r], par_r);
+                const T* sl = ring + slot_r * slot_elems + my_off;
 #pragma unroll
-                for (int j = 0; j < VY; ++j) vload<T, VX>(st.pl[0][NEW][j], sl + my_off + j * TX);
+                for (int j = 0; j < VY; ++j) pl[0][NEW].load_nat(j, sl + j * TX);
             }
-            // levels 1..D: level l computes plane r - l
+            const int rpar = r & 1;
+            // levels 1..D: level l computes plane z = r - l
 #pragma unroll
             for (int l = 1; l <= D; ++l) {
                 const int z = r - l;
-                const int lo = max(za - (D - l), zmin), hi = min(zb - 1 + (D - l), zmax);
-                if (z < lo || z > hi) continue;
-                const int zg = p.zbase + z;
-                const bool zfix = (zg == 0) || (zg == p.nzg - 1);
-                const T* top;
-                const T* bot;
-                if (l == 1) {
-                    uint32_t k = kbase + (z - rl0);
-                    const T* sl = ring + (k % ST7_RING) * slot_elems;
-                    top = sl + top_off;
-                    bot = sl + bot_off;
-                } else {
-                    const V* xb = xbuf + ((size_t)(l - 2) * 4 + (z & 1) * 2) * NT;
-                    top = reinterpret_cast<const T*>(xb + NT + tyu * NTX + st.tx);   // S-row of block above
-                    bot = reinterpret_cast<const T*>(xb + tyd * NTX + st.tx);        // N-row of block below
+                bool zfix = false;
+                if (!STEADY) {
+                    const int lo = max(za - (D - l), zmin), hi = min(zb - 1 + (D - l), zmax);
+                    if (z < lo || z > hi) continue;
+                    const int zg = p.zbase + z;
+                    zfix = (zg == 0) || (zg == p.nzg - 1);
                 }
+                const int zpar = rpar ^ (l & 1);
+                Row<T> top, bot;
+                if (l == 1) {   // level-0 neighbours of plane r-1 straight from the TMA ring
+                    const T* sl = ring + slot_m1 * slot_elems;
+                    top = row_nat(sl + top_off);
+                    bot = row_nat(sl + bot_off);
+                } else {        // rows exchanged by the blocks above / below in round r-1
+                    const int o = ((l - 2) * 4 + zpar * 2) * MAXT;
+                    top = row_x(xtop + o);
+                    bot = row_x(xbot + o);
+                }
+                B& dst = l < D ? pl[l < D ? l : 0][NEW] : outv;
+                if (!STEADY && zfix)
+                    st7_level<NTX, VY, EXACT>(pl[l - 1][PREV], pl[l - 1][CUR], pl[l - 1][NEW], top, bot,
+                                              Coef<T>::fixed(), yslow, rowfix, dst);
+                else
+                    st7_level<NTX, VY, EXACT>(pl[l - 1][PREV], pl[l - 1][CUR], pl[l - 1][NEW], top, bot, kc,
+                                              yslow, rowfix, dst);
                 if (l < D) {
-                    st.compute_level(st.pl[l - 1][PREV], st.pl[l - 1][CUR], st.pl[l - 1][NEW], top, bot, zfix,
-                                     st.pl[l][NEW]);
-                    V* xb = xbuf + ((size_t)(l - 1) * 4 + (z & 1) * 2) * NT;
-                    vstore<T, VX>(reinterpret_cast<T*>(xb + threadIdx.x), st.pl[l][NEW][0]);
-                    vstore<T, VX>(reinterpret_cast<T*>(xb + NT + threadIdx.x), st.pl[l][NEW][VY - 1]);
+                    V* xb = xw + ((l - 1) * 4 + zpar * 2) * MAXT;
+                    dst.store_x(0, xb);
+                    dst.store_x(VY - 1, xb + MAXT);
                 } else {
-                    st.compute_level(st.pl[l - 1][PREV], st.pl[l - 1][CUR], st.pl[l - 1][NEW], top, bot, zfix,
-                                     st.outv);
-                    const int xg = st.Lx + VX * st.tx;
-                    if (xg >= st.ox0 && xg < st.ox1) {
-                        T* base = outp + (size_t)z * plane + xg;
+                    T* base = outcol + (size_t)z * plane;
 #pragma unroll
-                        for (int j = 0; j < VY; ++j) {
-                            const int yg = st.Ly + VY * st.ty + j;
-                            if (yg >= st.oy0 && yg < st.oy1) gstore<T, VX>(base + (size_t)yg * p.nx, st.outv[j]);
-                        }
-                    }
+                    for (int j = 0; j < VY; ++j)
+                        if (rowmask & (1u << j)) outv.store_global(j, base + (size_t)j * p.nx);
                 }
             }
             __syncthreads();
+            // advance the ring cursors
+            slot_m1 = slot_r;
+            if (++slot_r == (uint32_t)RING) { slot_r = 0; par_r ^= 1; }
+            if (++slot_f == (uint32_t)RING) slot_f = 0;
+        };
+        auto any_round = [&](auto PHc, int r) {
+            if (r >= rs0 && r <= rs1) round(PHc, std::true_type{}, r);
+            else round(PHc, std::false_type{}, r);
         };
 
         for (int r = r0; r <= r1;) {
-            round(std::integral_constant<int, 0>{}, r);
+            any_round(std::integral_constant<int, 0>{}, r);
             if (++r > r1) break;
-            round(std::integral_constant<int, 1>{}, r);
+            any_round(std::integral_constant<int, 1>{}, r);
             if (++r > r1) break;
-            round(std::integral_constant<int, 2>{}, r);
+            any_round(std::integral_constant<int, 2>{}, r);
             ++r;
         }
     }
