@@ -63,10 +63,13 @@ static int encode_3d(CUtensorMap* map, const void* base, st_dtype dt, int nx, in
     cuuint64_t strides[2] = {(cuuint64_t)nx * E, (cuuint64_t)nx * ny * E};
     cuuint32_t box[3] = {(cuuint32_t)bx, (cuuint32_t)by, 1};
     cuuint32_t es[3] = {1, 1, 1};
+    // L2 promotion: the tile boxes start at arbitrary 16-byte offsets, so a
+    // 256-byte promotion would fetch up to twice the requested sectors
+    CUtensorMapL2promotion promo = CU_TENSOR_MAP_L2_PROMOTION_NONE;
+    if (const char* e = getenv("ST_L2PROMO")) promo = (CUtensorMapL2promotion)atoi(e);
     CUresult r = enc(map, dt == ST_F32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3,
                      const_cast<void*>(base), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                     CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                     CU_TENSOR_MAP_SWIZZLE_NONE, promo, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (r != CUDA_SUCCESS) return fail(ST_ECUDA, "cuTensorMapEncodeTiled failed (%d) box %dx%d", (int)r, bx, by);
     return ST_OK;
 }
@@ -118,8 +121,10 @@ static void variant_for(st_dtype dt, int d, int& vy, int& maxt) {
         int a = 0, b = 0;
         if (sscanf(e, "%dx%d", &a, &b) == 2) { vy = a; maxt = b; return; }
     }
-    if (dt == ST_F32) { vy = d <= 4 ? 2 : 2; maxt = d <= 4 ? 512 : 256; return; }
-    vy = 2; maxt = d <= 3 ? 512 : 256;
+    // measured on B200 (tools/quickbench.py): VY=4 / 256 threads is fastest
+    // while it fits without spills; deeper sweeps need the smaller block
+    if (dt == ST_F32) { vy = d <= 4 ? 4 : 2; maxt = 256; return; }
+    vy = d <= 3 ? 4 : 2; maxt = 256;
 }
 
 static St7LaunchFn lookup7(st_dtype dt, bool exact, int d, int vy, int maxt) {

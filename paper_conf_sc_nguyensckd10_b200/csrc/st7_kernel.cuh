@@ -75,8 +75,8 @@ template <int VY> struct Blk<float, VY> {
     __device__ __forceinline__ void store_x(int j, float4* s) const {   // exchange row, pair order
         *s = make_float4(a[j].x, a[j].y, b[j].x, b[j].y);
     }
-    __device__ __forceinline__ void store_global(int j, float* g) const {
-        st_global_v4(g, make_float4(a[j].x, b[j].x, a[j].y, b[j].y));
+    __device__ __forceinline__ void store_global(int j, float* g) const {  // plain store: predicable
+        *reinterpret_cast<float4*>(g) = make_float4(a[j].x, b[j].x, a[j].y, b[j].y);
     }
 };
 template <int VY> struct Blk<double, VY> {
@@ -87,7 +87,7 @@ template <int VY> struct Blk<double, VY> {
     }
     __device__ __forceinline__ void store_x(int j, double2* s) const { *s = make_double2(v[j][0], v[j][1]); }
     __device__ __forceinline__ void store_global(int j, double* g) const {
-        st_global_v2(g, make_double2(v[j][0], v[j][1]));
+        *reinterpret_cast<double2*>(g) = make_double2(v[j][0], v[j][1]);
     }
 };
 
@@ -312,6 +312,9 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
         uint32_t slot_r = kbase % RING, par_r = (kbase / RING) & 1;       // for plane r
         uint32_t slot_f = (kbase + PF) % RING;                            // for plane r + PF
         uint32_t slot_m1 = (slot_r + RING - 1) % RING;                    // for plane r - 1
+        // output row pointer of plane r - D (level D at round r), advanced by one plane per round
+        T* pout = outcol + (long long)(r0 - D) * (long long)plane;
+        const int nxs = p.nx;
 
         auto round = [&](auto PHc, auto STEADYc, int r) {
             constexpr int PH = decltype(PHc)::value;
@@ -365,13 +368,13 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                     dst.store_x(0, xb);
                     dst.store_x(VY - 1, xb + MAXT);
                 } else {
-                    T* base = outcol + (size_t)z * plane;
 #pragma unroll
                     for (int j = 0; j < VY; ++j)
-                        if (rowmask & (1u << j)) outv.store_global(j, base + (size_t)j * p.nx);
+                        if (rowmask & (1u << j)) outv.store_global(j, pout + j * nxs);
                 }
             }
             __syncthreads();
+            pout += plane;
             // advance the ring cursors
             slot_m1 = slot_r;
             if (++slot_r == (uint32_t)RING) { slot_r = 0; par_r ^= 1; }
