@@ -459,7 +459,7 @@ static int launch_lbm(st_plan* p, const void* src, void* dst, const uint8_t* fla
     else lid_coeffs<double>(p->lid, prm.lidc);
     const long long cells = (long long)(sv.zb - sv.za) * p->nx * p->ny;
     if (cells <= 0) return ST_OK;
-    const int grid = (int)std::min<long long>((cells + 255) / 256, (long long)p->sms * 16);
+    const int grid = (int)std::min<long long>((cells + 255) / 256, (long long)p->sms * (p->dtype == ST_F32 ? 4 : 3));
     cudaError_t e = lbm_push_launch(p->dtype == ST_F32 ? 0 : 1, p->exact, src, dst, flags, prm, grid,
                                     sv.stream ? sv.stream : p->stream);
     if (e != cudaSuccess) return fail(ST_ECUDA, "lbm launch: %s", cudaGetErrorString(e));

@@ -116,7 +116,7 @@ __device__ __forceinline__ void collide(T (&f)[19], T omega) {
 
 // dim_T = 1: push form, one thread per cell, grid-stride over the updated planes.
 template <typename T, bool E>
-__global__ void __launch_bounds__(256)
+__global__ void __launch_bounds__(256, (sizeof(T) == 4 ? 4 : 3))
 lbm_push_kernel(const T* __restrict__ src, T* __restrict__ dst, const uint8_t* __restrict__ flags,
                 const LbmParams p) {
     const size_t plane = (size_t)p.nx * p.ny;
