@@ -65,6 +65,7 @@ def _compile(src, obj, extra, verbose):
         cmd = [NVCC, *COMMON, *extra, "-x", "cu", "-c", os.path.join(CSRC, src), "-o", obj]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
+        cmd.insert(1, "-Xptxas=-warn-spills")
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"nvcc failed for {src}:\n{r.stderr[-6000:]}")
@@ -86,7 +87,8 @@ def build(force: bool = False, verbose: bool = False, jobs: int | None = None) -
             futs = {ex.submit(_compile, s, o, e, verbose): s for s, o, e in todo}
             for f in cf.as_completed(futs):
                 logs[futs[f]] = f.result()
-    if todo or not os.path.exists(LIB):
+    stale_lib = not os.path.exists(LIB) or any(os.path.getmtime(o) > os.path.getmtime(LIB) for o in objs)
+    if todo or stale_lib:
         tmp = LIB + f".tmp{os.getpid()}"
         cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-Xcompiler", "-fPIC"]
         r = subprocess.run(cmd, capture_output=True, text=True)

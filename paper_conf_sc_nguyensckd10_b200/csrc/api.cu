@@ -105,12 +105,18 @@ struct st_plan {
     int* d_count = nullptr;
     int* h_count = nullptr;
     const void* flags_checked = nullptr;
+    uint8_t* fl2 = nullptr;          // flags | 0x80 (FLUID next to non-FLUID), lbm_35d input
+    size_t fl2_bytes = 0;
+    const void* fl2_of = nullptr;
     // distribution (Z slabs)
     Dist dist;
     std::map<int, Geo7> geo7;  // by depth
 };
 
 static size_t esize(st_dtype d) { return d == ST_F32 ? 4 : 8; }
+struct GeoL { int TY = 0, wx = 0, wy = 0, tiles_x = 0, tiles_y = 0; size_t smem = 0; };
+static int planL(const st_plan* p, int d, GeoL& g);
+static int max_lbm_depth(const st_plan* p);
 
 // Kernel variant (rows per thread VY, max threads per CTA) for a sweep depth:
 // the register budget of each (D, VY, MAXT) instantiation, from ptxas -v
@@ -246,6 +252,7 @@ extern "C" void st_destroy(st_plan* p) {
     p->dist.destroy();
     for (void* b : p->hbuf) if (b) cudaFree(b);
     if (p->hflags) cudaFree(p->hflags);
+    if (p->fl2) cudaFree(p->fl2);
     if (p->d_count) cudaFree(p->d_count);
     if (p->h_count) cudaFreeHost(p->h_count);
     if (p->own_stream && p->stream) cudaStreamDestroy(p->stream);
@@ -294,10 +301,15 @@ extern "C" int st_plan_get_info(const st_plan* p, int lbm, st_plan_info* info) {
     if (!p || !info) return fail(ST_EINVAL, "NULL argument");
     memset(info, 0, sizeof *info);
     if (lbm) {
-        info->tile_x = p->nx; info->tile_y = p->ny; info->out_x = p->nx; info->out_y = p->ny;
-        info->tiles_x = info->tiles_y = 1; info->ctas = p->sms * 8; info->threads = 256; info->kappa = 1.0;
-        info->kernel = 100;
-        info->dim_t_sweep = 1;
+        const int d = max_lbm_depth(p);
+        GeoL g;
+        if (planL(p, d, g)) return ST_EUNSUPPORTED;
+        info->tile_x = 32; info->tile_y = g.TY; info->out_x = g.wx; info->out_y = g.wy;
+        info->tiles_x = g.tiles_x; info->tiles_y = g.tiles_y; info->ctas = p->sms; info->threads = 32 * g.TY;
+        info->smem_bytes = (int)g.smem;
+        info->kappa = (double)g.tiles_x * 32 * g.tiles_y * g.TY / ((double)p->nx * p->ny);
+        info->kernel = (d == 1 && getenv("ST_LBM_35D") == nullptr) ? 100 : 200 + d;
+        info->dim_t_sweep = d;
         return ST_OK;
     }
     auto it = p->geo7.find(p->dimK);
@@ -449,6 +461,51 @@ static void lid_coeffs(const double lid[3], double out[19]) {
     }
 }
 
+// LBM 3.5D geometry for sweep depth d: 32 x TY tiles, TY as large as the
+// (d-1) three-plane assembly rings allow in shared memory (<= 16 rows)
+static int planL(const st_plan* p, int d, GeoL& g) {
+    const size_t E = esize(p->dtype);
+    for (int ty = 16; ty >= 2; --ty) {
+        const size_t smem = (size_t)(d - 1) * 3 * 19 * 34 * (ty + 2) * E;
+        if (smem > p->smem_optin) continue;
+        if (ty - 2 * d < 1) break;
+        g.TY = ty; g.smem = smem;
+        g.wx = 32 - 2 * d; g.wy = ty - 2 * d;
+        g.tiles_x = (p->nx + g.wx - 1) / g.wx; g.tiles_y = (p->ny + g.wy - 1) / g.wy;
+        return ST_OK;
+    }
+    return fail(ST_EUNSUPPORTED, "LBM dim_T %d does not fit on chip", d);
+}
+
+static int max_lbm_depth(const st_plan* p) {
+    GeoL g;
+    for (int d = std::min(p->dimT, LBM35_MAX_D); d >= 1; --d)
+        if (planL(p, d, g) == ST_OK) return d;
+    return 1;
+}
+
+static int launch_lbm35(st_plan* p, const void* src, void* dst, int d, double omega, const SlabView& sv) {
+    GeoL g;
+    int rc = planL(p, d, g);
+    if (rc) return rc;
+    Lbm35Params prm{};
+    prm.src = src; prm.dst = dst; prm.fl2 = p->fl2 + sv.flags_off;
+    prm.nx = p->nx; prm.ny = p->ny; prm.nzb = sv.nzb; prm.zbase = sv.zbase; prm.nzg = p->nz;
+    prm.za = sv.za; prm.zb = sv.zb;
+    prm.tiles_x = g.tiles_x; prm.wx = g.wx; prm.wy = g.wy;
+    prm.work = (long long)g.tiles_x * g.tiles_y * (sv.zb - sv.za);
+    prm.omega = omega;
+    if (p->dtype == ST_F32) lid_coeffs<float>(p->lid, prm.lidc);
+    else lid_coeffs<double>(p->lid, prm.lidc);
+    if (prm.work <= 0) return ST_OK;
+    const int grid = (int)std::min<long long>(p->sms, prm.work);
+    cudaError_t e = lbm35_launch(p->dtype == ST_F32 ? 0 : 1, p->exact, d, prm, grid, 32 * g.TY, g.smem,
+                                 sv.stream ? sv.stream : p->stream);
+    if (e != cudaSuccess) return fail(ST_ECUDA, "lbm_35d launch (d=%d): %s", d, cudaGetErrorString(e));
+    ++p->launches;
+    return ST_OK;
+}
+
 static int launch_lbm(st_plan* p, const void* src, void* dst, const uint8_t* flags, double omega,
                       const SlabView& sv) {
     LbmParams prm{};
@@ -489,15 +546,31 @@ static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T
         CUDA_TRY(cudaMemcpyAsync(fdst, fsrc, n, cudaMemcpyDeviceToDevice, p->stream));
         return ST_OK;
     }
-    // dim_T = 1 push sweeps (the on-chip multi-level LBM sweep is lbm_35d)
+    // dim_T = 1: the fused push kernel (fastest measured on B200); dim_T >= 2:
+    // the on-chip multi-level sweep lbm_35d (ST_LBM_35D=1 forces it for dim_T = 1)
+    const bool push = max_lbm_depth(p) == 1 && getenv("ST_LBM_35D") == nullptr;
+    if (!push && p->fl2_of != flags) {   // neighbour-flag prepass (once per flags pointer)
+        const size_t cells = (size_t)p->nx * p->ny * p->dist.nzb;
+        if (p->fl2_bytes < cells) {
+            if (p->fl2) cudaFree(p->fl2);
+            p->fl2 = nullptr; p->fl2_bytes = 0;
+            if (cudaMalloc(&p->fl2, cells) != cudaSuccess) { cudaGetLastError(); return fail(ST_ENOMEM, "fl2"); }
+            p->fl2_bytes = cells;
+        }
+        cudaError_t e = lbm_fl2(flags, p->fl2, p->nx, p->ny, p->dist.nzb, p->stream);
+        if (e != cudaSuccess) return fail(ST_ECUDA, "fl2 prepass: %s", cudaGetErrorString(e));
+        p->fl2_of = flags;
+    }
+    std::vector<int> ds = push ? std::vector<int>(T, 1) : sweep_depths(T, max_lbm_depth(p));
     const void* src = fsrc;
     void* dst = fdst;
     void* bufs[2] = {fsrc, fdst};
-    const int S = T;
+    const int S = (int)ds.size();
     for (int s = 0; s < S; ++s) {
-        rc = p->dist.sweep(p->stream, 1, src, dst, 19 * esize(p->dtype), (size_t)p->nx * p->ny,
+        rc = p->dist.sweep(p->stream, ds[s], src, dst, 19 * esize(p->dtype), (size_t)p->nx * p->ny,
                            [&](const void* a, void* b, const SlabView& sv) {
-                               return launch_lbm(p, a, b, flags + (sv.flags_off), omega, sv);
+                               if (push) return launch_lbm(p, a, b, flags + (sv.flags_off), omega, sv);
+                               return launch_lbm35(p, a, b, ds[s], omega, sv);
                            });
         if (rc) return rc;
         src = bufs[(s + 1) % 2];
@@ -534,6 +607,7 @@ extern "C" int lbm_d3q19_run(st_plan* p, void* fsrc, void* fdst, double omega, i
     CUDA_TRY(cudaMemcpyAsync(p->hbuf[0], fsrc, n, cudaMemcpyHostToDevice, p->stream));
     CUDA_TRY(cudaMemcpyAsync(p->hflags, flags, cells, cudaMemcpyHostToDevice, p->stream));
     p->flags_checked = nullptr;  // staging buffer content changes per call
+    p->fl2_of = nullptr;
     rc = runlbm_device(p, p->hbuf[0], p->hbuf[1], omega, T, p->hflags);
     if (rc) return rc;
     CUDA_TRY(cudaMemcpyAsync(fdst, p->hbuf[1], n, cudaMemcpyDeviceToHost, p->stream));

@@ -18,6 +18,56 @@ cudaError_t lbm_push_launch(int dtype, bool exact, const void* src, void* dst, c
                  : push_t<double, false>(src, dst, flags, p, grid, s);
 }
 
+template <typename T, int D, bool E>
+static cudaError_t l35_t(const Lbm35Params& p, int grid, int threads, size_t smem, cudaStream_t s) {
+    auto k = lbm_35d_kernel<T, D, E>;
+    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    k<<<grid, threads, smem, s>>>(p);
+    return cudaGetLastError();
+}
+
+template <typename T, bool E>
+static cudaError_t l35_d(int D, const Lbm35Params& p, int grid, int threads, size_t smem, cudaStream_t s) {
+    switch (D) {
+        case 1: return l35_t<T, 1, E>(p, grid, threads, smem, s);
+        case 2: return l35_t<T, 2, E>(p, grid, threads, smem, s);
+        case 3: return l35_t<T, 3, E>(p, grid, threads, smem, s);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+cudaError_t lbm35_launch(int dtype, bool exact, int D, const Lbm35Params& p, int grid, int threads, size_t smem,
+                         cudaStream_t s) {
+    if (dtype == 0) return exact ? l35_d<float, true>(D, p, grid, threads, smem, s)
+                                 : l35_d<float, false>(D, p, grid, threads, smem, s);
+    return exact ? l35_d<double, true>(D, p, grid, threads, smem, s) : l35_d<double, false>(D, p, grid, threads, smem, s);
+}
+
+// fl2 = flags | 0x80 where a FLUID cell has a non-FLUID (or out-of-lattice) neighbour
+__global__ void lbm_fl2_kernel(const uint8_t* __restrict__ flags, uint8_t* __restrict__ fl2, int nx, int ny, int nz) {
+    const size_t plane = (size_t)nx * ny, n = plane * nz;
+    for (size_t c = blockIdx.x * (size_t)blockDim.x + threadIdx.x; c < n; c += (size_t)gridDim.x * blockDim.x) {
+        const int x = (int)(c % nx), y = (int)((c / nx) % ny), z = (int)(c / plane);
+        uint8_t f = flags[c];
+        if (f == 0) {
+            bool nb = false;
+            for (int i = 1; i < 19; ++i) {
+                const int X = x + c_ex[i], Y = y + c_ey[i], Z = z + c_ez[i];
+                if (X < 0 || Y < 0 || Z < 0 || X >= nx || Y >= ny || Z >= nz) { nb = true; break; }
+                if (flags[(size_t)Z * plane + (size_t)Y * nx + X] != 0) { nb = true; break; }
+            }
+            if (nb) f |= 0x80;
+        }
+        fl2[c] = f;
+    }
+}
+
+cudaError_t lbm_fl2(const uint8_t* flags, uint8_t* fl2, int nx, int ny, int nz, cudaStream_t s) {
+    lbm_fl2_kernel<<<148 * 8, 256, 0, s>>>(flags, fl2, nx, ny, nz);
+    return cudaGetLastError();
+}
+
 // counts FLUID cells on the 6 faces of the lattice (the GPU path needs 0)
 __global__ void shell_check_kernel(const uint8_t* __restrict__ flags, int nx, int ny, int nz, int* count) {
     const long long nxy = (long long)nx * ny;

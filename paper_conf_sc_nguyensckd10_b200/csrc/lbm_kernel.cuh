@@ -158,4 +158,158 @@ lbm_push_kernel(const T* __restrict__ src, T* __restrict__ dst, const uint8_t* _
     }
 }
 
+// ---------------------------------------------------------------------------
+// lbm_35d_kernel: the 3.5D-blocked D3Q19 sweep (dim_T = D levels on chip).
+//
+// A CTA owns a 32 x TY cell tile (one cell per thread, a warp = one row) of
+// an XY sub-plane and streams it along Z.  Transition l (level
+// l-1 -> l) at round r takes the level-(l-1) plane q = r-l+1, collides every
+// FLUID cell (BGK, X9) and PUSHES the 19 post-collision values
+// into level l's planes q-1, q, q+1; a push into a WALL / LID cell bounces
+// back into the cell's own opposite population (X10).  Level l's plane r-l is
+// then complete (its three source planes were processed in rounds r-2..r),
+// so lag 1 per level and one barrier per transition.  Levels 1..D-1 are
+// assembled in a 3-plane shared-memory ring per level (padded by one cell so
+// edge pushes stay in bounds); the last transition pushes straight into the
+// output lattice, only for target cells in the tile's written region
+// (X - 2D) x (Y - 2D) and the segment's planes, so every (cell, population)
+// of f_dst is written exactly once.  Level 0 is read with coalesced SoA loads,
+// prefetched one plane ahead into registers.
+// fl2 = flags | 0x80 for a FLUID cell with a non-FLUID neighbour (host prepass):
+// only those cells look at their neighbours' flags.
+// ---------------------------------------------------------------------------
+struct Lbm35Params {
+    const void* src;
+    void* dst;
+    const uint8_t* fl2;
+    int nx, ny, nzb, zbase, nzg, za, zb;
+    int tiles_x, wx, wy;
+    long long work;
+    double omega;
+    double lidc[19];
+};
+
+template <int I, typename T, bool E, typename F>
+__device__ __forceinline__ void lbm_push_one(const T (&fs)[19], uint32_t fl, int x, int y, int q, int nx, int ny,
+                                             size_t plane, const uint8_t* __restrict__ fl2, const T* lidc, F&& put) {
+    constexpr int ex = D3Q19<I>::ex, ey = D3Q19<I>::ey, ez = D3Q19<I>::ez;
+    if constexpr (I == 0) {
+        put(0, 0, 0, 0, fs[0]);
+    } else {
+        uint32_t tf = 0;
+        if (fl & 0x80u) tf = __ldg(fl2 + (size_t)(q + ez) * plane + (size_t)(y + ey) * nx + (x + ex)) & 0x7fu;
+        if (tf == 0) put(I, ex, ey, ez, fs[I]);
+        else if (tf == 1) put(D3Q19<I>::opp, 0, 0, 0, fs[I]);
+        else put(D3Q19<I>::opp, 0, 0, 0, Ar<T, E>::sub(fs[I], lidc[I]));
+    }
+}
+
+template <typename T, int D, bool E>
+__global__ void __launch_bounds__(512, 1) lbm_35d_kernel(const Lbm35Params p) {
+    constexpr int TX = 32, PX = TX + 2;
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+    const int TY = blockDim.x >> 5, PY = TY + 2;
+    const int pstride = PX * PY;                 // one population plane of the padded tile
+    const int sstride = 19 * pstride;            // one ring slot
+    T* asmb = reinterpret_cast<T*>(smem_raw);    // [D-1][3][19][PY][PX]
+    const T* __restrict__ src = static_cast<const T*>(p.src);
+    T* __restrict__ dst = static_cast<T*>(p.dst);
+    const size_t plane = (size_t)p.nx * p.ny;
+    const size_t nc = plane * p.nzb;
+    const T omega = T(p.omega);
+    T lidc[19];
+#pragma unroll
+    for (int i = 0; i < 19; ++i) lidc[i] = T(p.lidc[i]);
+    const int zmin = max(0, -p.zbase);
+    const int zmax = min(p.nzb - 1, p.nzg - 1 - p.zbase);
+    const int nzo = p.zb - p.za;
+    const long long G = gridDim.x;
+    long long item = p.work * (long long)blockIdx.x / G;
+    const long long item_end = p.work * ((long long)blockIdx.x + 1) / G;
+    const int me = (ty + 1) * PX + (tx + 1);     // my cell in a padded population plane
+
+    while (item < item_end) {
+        const int tile = (int)(item / nzo);
+        const long long seg_end = min(item_end, (long long)(tile + 1) * nzo);
+        const int za = p.za + (int)(item - (long long)tile * nzo);
+        const int zb = p.za + (int)(seg_end - (long long)tile * nzo);
+        item = seg_end;
+        const int ix = tile % p.tiles_x, iy = tile / p.tiles_x;
+        const int ox0 = ix * p.wx, ox1 = min(ox0 + p.wx, p.nx);
+        const int oy0 = iy * p.wy, oy1 = min(oy0 + p.wy, p.ny);
+        const int x = ox0 - D + tx, y = oy0 - D + ty;
+        const bool inb = x >= 0 && x < p.nx && y >= 0 && y < p.ny;
+        const size_t cxy = inb ? (size_t)y * p.nx + x : 0;
+        const int rl0 = max(za - D, zmin), rl1 = min(zb - 1 + D, zmax);
+
+        T fnext[19];
+        uint32_t flnext = 0;
+        auto load = [&](int q) {
+            if (inb && q <= rl1) {
+                const size_t c = (size_t)q * plane + cxy;
+#pragma unroll
+                for (int i = 0; i < 19; ++i) fnext[i] = src[i * nc + c];
+                flnext = p.fl2[c];
+            }
+        };
+        load(rl0);
+        uint64_t flh = 0;   // own flags of the last 8 level-0 planes (byte k = plane r-k)
+
+        for (int r = rl0; r <= zb - 1 + D; ++r) {
+            T f[19];
+#pragma unroll
+            for (int i = 0; i < 19; ++i) f[i] = fnext[i];
+            flh = (flh << 8) | (r <= rl1 ? flnext : 0u);
+            load(r + 1);
+#pragma unroll
+            for (int l = 1; l <= D; ++l) {
+                const int q = r - l + 1;                                 // level-(l-1) plane processed
+                const int lo = max(za - D + l - 1, zmin), hi = min(zb + D - l, zmax);
+                if (q >= lo && q <= hi && inb) {
+                    if (l > 1) {   // level l-1 plane q from the assembly ring
+                        const T* a = asmb + ((size_t)(l - 2) * 3 + (size_t)(q % 3)) * sstride + me;
+#pragma unroll
+                        for (int i = 0; i < 19; ++i) f[i] = a[i * pstride];
+                    }
+                    const uint32_t fl = (uint32_t)(flh >> (8 * (l - 1))) & 0xffu;
+                    if (l < D) {
+                        T* ab = asmb + (size_t)(l - 1) * 3 * sstride;
+                        auto put = [&](int pop, int ex, int ey, int ez, T v) {
+                            ab[(size_t)((q + ez + 3) % 3) * sstride + pop * pstride + me + ey * PX + ex] = v;
+                        };
+                        if ((fl & 0x7fu) != 0) {
+#pragma unroll
+                            for (int i = 0; i < 19; ++i) put(i, 0, 0, 0, f[i]);
+                        } else {
+                            collide<T, E>(f, omega);
+                            [&]<int... Is>(std::integer_sequence<int, Is...>) {
+                                (lbm_push_one<Is, T, E>(f, fl, x, y, q, p.nx, p.ny, plane, p.fl2, lidc, put), ...);
+                            }(std::make_integer_sequence<int, 19>{});
+                        }
+                    } else {
+                        const size_t cq = (size_t)q * plane + cxy;
+                        auto put = [&](int pop, int ex, int ey, int ez, T v) {
+                            const int tx2 = x + ex, ty2 = y + ey, tz = q + ez;
+                            if (tx2 >= ox0 && tx2 < ox1 && ty2 >= oy0 && ty2 < oy1 && tz >= za && tz < zb)
+                                dst[pop * nc + (size_t)((long long)cq + ex + (long long)ey * p.nx +
+                                                        (long long)ez * (long long)plane)] = v;
+                        };
+                        if ((fl & 0x7fu) != 0) {
+#pragma unroll
+                            for (int i = 0; i < 19; ++i) put(i, 0, 0, 0, f[i]);
+                        } else {
+                            collide<T, E>(f, omega);
+                            [&]<int... Is>(std::integer_sequence<int, Is...>) {
+                                (lbm_push_one<Is, T, E>(f, fl, x, y, q, p.nx, p.ny, plane, p.fl2, lidc, put), ...);
+                            }(std::make_integer_sequence<int, 19>{});
+                        }
+                    }
+                }
+                if (D > 1) __syncthreads();
+            }
+        }
+    }
+}
+
 }  // namespace st35d

@@ -34,17 +34,38 @@ def run_gpu(f0, flags, omega, T, dim_T=1, exact=False, lid=(0.05, 0.0, 0.0)):
 
 
 @pytest.mark.parametrize("dtype", [np.float32, np.float64])
-@pytest.mark.parametrize("shape", [(32, 24, 20), (64, 40, 9), (16, 16, 16)])
-def test_cavity_random(oracle_lib, dtype, shape):
+@pytest.mark.parametrize("shape", [(32, 24, 20), (64, 40, 9), (16, 16, 16), (96, 50, 13)])
+@pytest.mark.parametrize("dim_T", [1, 2, 3])
+def test_cavity_random(oracle_lib, dtype, shape, dim_T):
     nx, ny, nz = shape
     flags = stgen.cavity_flags(nx, ny, nz)
     f0 = stgen.lbm_random(nx, ny, nz, 3, dtype)
-    T = 5
+    T = 7
     ref = oracle_lib.lbm(f0, flags, 1.6, T)
-    got = run_gpu(f0, flags, 1.6, T, exact=True)
+    got = run_gpu(f0, flags, 1.6, T, dim_T=dim_T, exact=True)
     assert np.array_equal(got, ref)
-    got = run_gpu(f0, flags, 1.6, T)
+    got = run_gpu(f0, flags, 1.6, T, dim_T=dim_T)
     assert relerr(got, ref) <= TOL[dtype]
+
+
+def test_obstacle_interior(oracle_lib):
+    # an interior WALL block: neighbour-flag slow path away from the shell
+    nx, ny, nz = 40, 30, 20
+    flags = stgen.cavity_flags(nx, ny, nz)
+    flags[8:12, 10:15, 12:20] = stgen.WALL
+    flags[5, 20, 30] = stgen.LID
+    f0 = stgen.lbm_random(nx, ny, nz, 9, np.float32)
+    ref = oracle_lib.lbm(f0, flags, 1.2, 6)
+    for d in (1, 2, 3):
+        assert np.array_equal(run_gpu(f0, flags, 1.2, 6, dim_T=d, exact=True), ref), d
+
+
+def test_dimT_invariance_lbm():
+    nx, ny, nz = 64, 36, 24
+    flags = stgen.cavity_flags(nx, ny, nz)
+    f0 = stgen.lbm_random(nx, ny, nz, 5, np.float32)
+    outs = [run_gpu(f0, flags, 1.6, 9, dim_T=d, exact=True) for d in (1, 2, 3)]
+    assert np.array_equal(outs[0], outs[1]) and np.array_equal(outs[0], outs[2])
 
 
 def test_T0_and_rest(oracle_lib):
