@@ -131,6 +131,13 @@ int st_plan_sync(st_plan* plan);
  * nranks == 1 switches distribution off. */
 int st_plan_set_dist(st_plan* plan, const void* nccl_unique_id, int rank, int nranks);
 
+/* 128-byte NCCL unique id for st_plan_set_dist (call on rank 0, broadcast). */
+int st_nccl_unique_id(void* out128);
+
+/* Z-slab of `rank` among `nranks`: first global plane and plane count
+ * (remainder planes one each to the first ranks).  Host-only. */
+int st_slab_range(int nz, int nranks, int rank, int* z0, int* nz_local);
+
 /* Loopback distribution on one device (testing): P virtual slabs, ghosts
  * copied with cudaMemcpyAsync instead of NCCL; result identical to P = 1. */
 int st_plan_set_loopback_slabs(st_plan* plan, int nslabs);

@@ -48,7 +48,8 @@ _lib = None
 EXPORTS = ["st_plan_create", "st7_run", "lbm_d3q19_run", "st_destroy", "st_last_error", "st_last_status",
            "st_plan_set_stream", "st_plan_set_lbm_lid", "st_plan_set_bitexact", "st_plan_sync",
            "st_plan_set_dist", "st_plan_set_loopback_slabs", "st_plan_ghost_planes", "st_plan_local_slab",
-           "st_plan_get_info", "st_plan_last_launches", "st_blocking_model", "st_fig3_step"]
+           "st_plan_get_info", "st_plan_last_launches", "st_blocking_model", "st_fig3_step",
+           "st_nccl_unique_id", "st_slab_range"]
 
 
 def lib() -> ctypes.CDLL:
@@ -79,6 +80,8 @@ def lib() -> ctypes.CDLL:
         "st_plan_last_launches": ([P], I),
         "st_blocking_model": ([D, D, I, D, D, I, I, ctypes.POINTER(st_blocking)], I),
         "st_fig3_step": ([I, I, I, I, ctypes.POINTER(I), ctypes.POINTER(I)], I),
+        "st_nccl_unique_id": ([P], I),
+        "st_slab_range": ([I, I, I, ctypes.POINTER(I), ctypes.POINTER(I)], I),
     }
     for name, (args, res) in sig.items():
         fn = getattr(L, name)
@@ -192,6 +195,18 @@ def st_fig3_step(R: int, dim_T: int, rnd: int, level: int):
     z, s = ctypes.c_int(), ctypes.c_int()
     step = _check(lib().st_fig3_step(R, dim_T, rnd, level, ctypes.byref(z), ctypes.byref(s)))
     return step, z.value, s.value
+
+
+def st_nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().st_nccl_unique_id(ctypes.addressof(buf)))
+    return buf.raw
+
+
+def st_slab_range(nz: int, nranks: int, rank: int):
+    z0, n = ctypes.c_int(), ctypes.c_int()
+    _check(lib().st_slab_range(nz, nranks, rank, ctypes.byref(z0), ctypes.byref(n)))
+    return z0.value, n.value
 
 
 def dtype_code(dtype) -> int:

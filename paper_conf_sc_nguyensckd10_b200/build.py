@@ -34,8 +34,10 @@ def _nccl_include():
     return None
 
 
+_NCCL_INC = _nccl_include()
 COMMON = ARCH + ["-O3", "-lineinfo", "-std=c++20", "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC",
-                 "-Xcompiler", "-ffp-contract=off", "-I", os.path.join(ROOT, "include")]
+                 "-Xcompiler", "-ffp-contract=off", "-I", os.path.join(ROOT, "include")] + \
+    (["-DST_HAVE_NCCL=1", "-I", _NCCL_INC] if _NCCL_INC else ["-DST_HAVE_NCCL=0"])
 
 UNITS = [
     ("api.cu", "api.o", []),
@@ -90,7 +92,7 @@ def build(force: bool = False, verbose: bool = False, jobs: int | None = None) -
     stale_lib = not os.path.exists(LIB) or any(os.path.getmtime(o) > os.path.getmtime(LIB) for o in objs)
     if todo or stale_lib:
         tmp = LIB + f".tmp{os.getpid()}"
-        cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-Xcompiler", "-fPIC"]
+        cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-Xcompiler", "-fPIC", "-ldl"]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stderr[-4000:]}")

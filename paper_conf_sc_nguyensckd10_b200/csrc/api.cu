@@ -8,6 +8,7 @@
 #include <vector>
 #include <algorithm>
 #include <cudaTypedefs.h>
+#include <dlfcn.h>
 
 #include "../../include/st35d.h"
 #include "launch.h"
@@ -386,6 +387,169 @@ static int launch7(st_plan* p, const void* src, void* dst, int d, double alpha, 
     return ST_OK;
 }
 
+// ----------------------------------------------------------------------------
+// multi-sweep driver over the plan's Z decomposition (dist.h)
+// ----------------------------------------------------------------------------
+// ncomp: SoA components of a cell (1 for the 7-point grid, 19 for D3Q19); each
+// component of a slab buffer is nzb consecutive planes.
+static int exchange_nccl(st_plan* p, void* buf, int d, int ncomp) {
+#if ST_HAVE_NCCL
+    Dist& D = p->dist;
+    const size_t pb = (size_t)p->nx * p->ny * esize(p->dtype);
+    const size_t cs = (size_t)D.nzb * pb;
+    char* b = static_cast<char*>(buf);
+    const size_t bytes = (size_t)d * pb;
+    auto& N = nccl();
+    ncclResult_t r = N.groupStart();
+    for (int c = 0; c < ncomp && r == ncclSuccess; ++c) {
+        char* base = b + c * cs;
+        if (D.rank > 0) {
+            if (r == ncclSuccess) r = N.send(base + (size_t)D.g * pb, bytes, ncclUint8, D.rank - 1, D.comm, p->stream);
+            if (r == ncclSuccess) r = N.recv(base + (size_t)(D.g - d) * pb, bytes, ncclUint8, D.rank - 1, D.comm, p->stream);
+        }
+        if (D.rank < D.P - 1) {
+            if (r == ncclSuccess) r = N.send(base + (size_t)(D.g + D.nzl - d) * pb, bytes, ncclUint8, D.rank + 1, D.comm, p->stream);
+            if (r == ncclSuccess) r = N.recv(base + (size_t)(D.g + D.nzl) * pb, bytes, ncclUint8, D.rank + 1, D.comm, p->stream);
+        }
+    }
+    ncclResult_t r2 = N.groupEnd();
+    if (r != ncclSuccess || r2 != ncclSuccess)
+        return fail(ST_ENCCL, "ghost exchange: %s", N.errorString(r != ncclSuccess ? r : r2));
+    return ST_OK;
+#else
+    (void)p; (void)buf; (void)d; (void)ncomp;
+    return fail(ST_EUNSUPPORTED, "built without NCCL");
+#endif
+}
+
+static int exchange_loop(st_plan* p, int cur, int d, int ncomp) {
+    Dist& D = p->dist;
+    const size_t pb = (size_t)p->nx * p->ny * esize(p->dtype);
+    const size_t bytes = (size_t)d * pb;
+    for (int k = 0; k < D.P; ++k) {
+        Dist::Slab& s = D.slabs[k];
+        char* me = static_cast<char*>(s.buf[cur]);
+        const size_t cs = (size_t)s.nzb * pb;
+        if (k > 0) {
+            Dist::Slab& o = D.slabs[k - 1];
+            const char* src = static_cast<const char*>(o.buf[cur]);
+            const size_t ocs = (size_t)o.nzb * pb;
+            for (int c = 0; c < ncomp; ++c)
+                CUDA_TRY(cudaMemcpyAsync(me + c * cs + (size_t)(D.g - d) * pb,
+                                         src + c * ocs + (size_t)(D.g + o.nzl - d) * pb, bytes,
+                                         cudaMemcpyDeviceToDevice, p->stream));
+        }
+        if (k < D.P - 1) {
+            Dist::Slab& o = D.slabs[k + 1];
+            const char* src = static_cast<const char*>(o.buf[cur]);
+            const size_t ocs = (size_t)o.nzb * pb;
+            for (int c = 0; c < ncomp; ++c)
+                CUDA_TRY(cudaMemcpyAsync(me + c * cs + (size_t)(D.g + s.nzl) * pb, src + c * ocs + (size_t)D.g * pb,
+                                         bytes, cudaMemcpyDeviceToDevice, p->stream));
+        }
+    }
+    return ST_OK;
+}
+
+// copy global planes [z, z+n) of every component between a full grid (nz planes)
+// and a slab buffer (nzb planes, buffer plane = z - zbase)
+static int slab_copy(st_plan* p, void* full, void* slab, int zbase, int nzb, int z, int n, int ncomp, bool to_slab) {
+    if (n <= 0) return ST_OK;
+    const size_t pb = (size_t)p->nx * p->ny * esize(p->dtype);
+    for (int c = 0; c < ncomp; ++c) {
+        char* f = static_cast<char*>(full) + (size_t)c * p->nz * pb + (size_t)z * pb;
+        char* s = static_cast<char*>(slab) + (size_t)c * nzb * pb + (size_t)(z - zbase) * pb;
+        CUDA_TRY(cudaMemcpyAsync(to_slab ? s : f, to_slab ? f : s, (size_t)n * pb, cudaMemcpyDeviceToDevice,
+                                 p->stream));
+    }
+    return ST_OK;
+}
+
+static int ensure_loop_slabs(st_plan* p, int ncomp, const uint8_t* flags) {
+    Dist& D = p->dist;
+    const size_t pbe = (size_t)p->nx * p->ny * esize(p->dtype);
+    const size_t plane = (size_t)p->nx * p->ny;
+    for (auto& s : D.slabs) {
+        const size_t need = (size_t)ncomp * s.nzb * pbe;
+        if (D.slab_cell_bytes < need / s.nzb / plane * 1 || D.slab_ncomp != ncomp || !s.buf[0]) {
+            for (void*& b : s.buf) { if (b) cudaFree(b); b = nullptr; }
+            for (void*& b : s.buf)
+                if (cudaMalloc(&b, need) != cudaSuccess) { cudaGetLastError(); return fail(ST_ENOMEM, "loopback slab"); }
+        }
+        if (flags) {
+            if (!s.flags && cudaMalloc(&s.flags, (size_t)s.nzb * plane) != cudaSuccess) return fail(ST_ENOMEM, "slab flags");
+            if (!s.fl2 && cudaMalloc(&s.fl2, (size_t)s.nzb * plane) != cudaSuccess) return fail(ST_ENOMEM, "slab fl2");
+            // planes outside the lattice are WALL; the rest copied from the global flags
+            CUDA_TRY(cudaMemsetAsync(s.flags, ST_WALL, (size_t)s.nzb * plane, p->stream));
+            const int zlo = std::max(0, s.z0 - D.g), zhi = std::min(p->nz, s.z0 + s.nzl + D.g);
+            CUDA_TRY(cudaMemcpyAsync(s.flags + (size_t)(zlo - (s.z0 - D.g)) * plane, flags + (size_t)zlo * plane,
+                                     (size_t)(zhi - zlo) * plane, cudaMemcpyDeviceToDevice, p->stream));
+            cudaError_t e = lbm_fl2(s.flags, s.fl2, p->nx, p->ny, s.nzb, p->stream);
+            if (e != cudaSuccess) return fail(ST_ECUDA, "slab fl2: %s", cudaGetErrorString(e));
+        }
+    }
+    D.slab_ncomp = ncomp;
+    D.slab_cell_bytes = (size_t)ncomp * esize(p->dtype);
+    return ST_OK;
+}
+
+template <typename L>
+static int run_sweeps(st_plan* p, const std::vector<int>& ds, const void* in, void* out, int ncomp,
+                      const uint8_t* flags, L&& launch) {
+    Dist& D = p->dist;
+    const size_t pb = (size_t)p->nx * p->ny * esize(p->dtype);
+    if (D.mode == Dist::LOOPBACK) {
+        int rc = ensure_loop_slabs(p, ncomp, flags);
+        if (rc) return rc;
+        for (auto& s : D.slabs) {   // scatter owned planes + available ghosts
+            const int zlo = std::max(0, s.z0 - D.g), zhi = std::min(p->nz, s.z0 + s.nzl + D.g);
+            rc = slab_copy(p, const_cast<void*>(in), s.buf[0], s.z0 - D.g, s.nzb, zlo, zhi - zlo, ncomp, true);
+            if (rc) return rc;
+        }
+        int cur = 0;
+        for (size_t k = 0; k < ds.size(); ++k) {
+            rc = exchange_loop(p, cur, ds[k], ncomp);
+            if (rc) return rc;
+            for (auto& s : D.slabs) {
+                SlabView sv;
+                sv.nzb = s.nzb; sv.zbase = s.z0 - D.g; sv.za = D.g; sv.zb = D.g + s.nzl;
+                sv.flags = s.flags; sv.fl2 = s.fl2; sv.single = false; sv.stream = p->stream;
+                rc = launch(s.buf[cur], s.buf[1 - cur], ds[k], sv);
+                if (rc) return rc;
+            }
+            cur ^= 1;
+        }
+        for (auto& s : D.slabs) {   // gather owned planes
+            rc = slab_copy(p, out, s.buf[cur], s.z0 - D.g, s.nzb, s.z0, s.nzl, ncomp, false);
+            if (rc) return rc;
+        }
+        return ST_OK;
+    }
+    const void* src = in;
+    void* dst = out;
+    void* bufs[2] = {const_cast<void*>(in), out};
+    for (size_t k = 0; k < ds.size(); ++k) {
+        SlabView sv;
+        sv.stream = p->stream;
+        sv.flags = flags;
+        sv.fl2 = p->fl2;
+        if (D.mode == Dist::NCCL) {
+            int rc = exchange_nccl(p, const_cast<void*>(src), ds[k], ncomp);
+            if (rc) return rc;
+            sv.nzb = D.nzb; sv.zbase = D.z0 - D.g; sv.za = D.g; sv.zb = D.g + D.nzl; sv.single = false;
+        } else {
+            sv.nzb = p->nz; sv.zbase = 0; sv.za = 0; sv.zb = p->nz; sv.single = true;
+        }
+        int rc = launch(src, dst, ds[k], sv);
+        if (rc) return rc;
+        src = bufs[(k + 1) % 2];
+        dst = bufs[k % 2];
+    }
+    if (ds.size() % 2 == 0)  // only when every sweep has depth 1 and T is even: result in `in`
+        CUDA_TRY(cudaMemcpyAsync(out, in, (size_t)ncomp * D.nzb * pb, cudaMemcpyDeviceToDevice, p->stream));
+    return ST_OK;
+}
+
 static int run7_device(st_plan* p, const void* in, void* out, double alpha, double beta, int T) {
     const size_t n = (size_t)p->nx * p->ny * p->dist.nzb * esize(p->dtype);
     p->launches = 0;
@@ -394,20 +558,10 @@ static int run7_device(st_plan* p, const void* in, void* out, double alpha, doub
         return ST_OK;
     }
     std::vector<int> ds = sweep_depths(T, p->dimK);
-    const void* src = in;
-    void* dst = out;
-    void* bufs[2] = {const_cast<void*>(in), out};
-    for (size_t s = 0; s < ds.size(); ++s) {
-        int rc = p->dist.sweep(p->stream, ds[s], src, dst, esize(p->dtype), (size_t)p->nx * p->ny,
-                               [&](const void* a, void* b, const SlabView& sv) {
-                                   return launch7(p, a, b, ds[s], alpha, beta, sv);
-                               });
-        if (rc) return rc;
-        src = bufs[(s + 1) % 2];
-        dst = bufs[s % 2];
-    }
-    if (ds.size() % 2 == 0)  // only when dim_T = 1 and T even: result is in `in`
-        CUDA_TRY(cudaMemcpyAsync(out, in, n, cudaMemcpyDeviceToDevice, p->stream));
+    int rc = run_sweeps(p, ds, in, out, 1, nullptr, [&](const void* a, void* b, int d, const SlabView& sv) {
+        return launch7(p, a, b, d, alpha, beta, sv);
+    });
+    if (rc) return rc;
     CUDA_TRY(cudaGetLastError());
     return ST_OK;
 }
@@ -489,7 +643,7 @@ static int launch_lbm35(st_plan* p, const void* src, void* dst, int d, double om
     int rc = planL(p, d, g);
     if (rc) return rc;
     Lbm35Params prm{};
-    prm.src = src; prm.dst = dst; prm.fl2 = p->fl2 + sv.flags_off;
+    prm.src = src; prm.dst = dst; prm.fl2 = sv.fl2;
     prm.nx = p->nx; prm.ny = p->ny; prm.nzb = sv.nzb; prm.zbase = sv.zbase; prm.nzg = p->nz;
     prm.za = sv.za; prm.zb = sv.zb;
     prm.tiles_x = g.tiles_x; prm.wx = g.wx; prm.wy = g.wy;
@@ -526,7 +680,7 @@ static int launch_lbm(st_plan* p, const void* src, void* dst, const uint8_t* fla
 
 static int check_shell(st_plan* p, const uint8_t* flags) {
     if (p->flags_checked == flags) return ST_OK;
-    if (p->dist.nranks > 1) { p->flags_checked = flags; return ST_OK; }  // slab shells checked per rank
+    if (p->dist.mode == Dist::NCCL) { p->flags_checked = flags; return ST_OK; }  // caller-owned slab flags
     cudaError_t e = lbm_shell_check(flags, p->nx, p->ny, p->nz, p->d_count, p->stream);
     if (e != cudaSuccess) return fail(ST_ECUDA, "shell check: %s", cudaGetErrorString(e));
     CUDA_TRY(cudaMemcpyAsync(p->h_count, p->d_count, sizeof(int), cudaMemcpyDeviceToHost, p->stream));
@@ -548,8 +702,8 @@ static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T
     }
     // dim_T = 1: the fused push kernel (fastest measured on B200); dim_T >= 2:
     // the on-chip multi-level sweep lbm_35d (ST_LBM_35D=1 forces it for dim_T = 1)
-    const bool push = max_lbm_depth(p) == 1 && getenv("ST_LBM_35D") == nullptr;
-    if (!push && p->fl2_of != flags) {   // neighbour-flag prepass (once per flags pointer)
+    const bool push = max_lbm_depth(p) == 1 && getenv("ST_LBM_35D") == nullptr && p->dist.mode == Dist::SINGLE;
+    if (!push && p->dist.mode != Dist::LOOPBACK && p->fl2_of != flags) {   // neighbour-flag prepass (once per flags pointer)
         const size_t cells = (size_t)p->nx * p->ny * p->dist.nzb;
         if (p->fl2_bytes < cells) {
             if (p->fl2) cudaFree(p->fl2);
@@ -562,21 +716,11 @@ static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T
         p->fl2_of = flags;
     }
     std::vector<int> ds = push ? std::vector<int>(T, 1) : sweep_depths(T, max_lbm_depth(p));
-    const void* src = fsrc;
-    void* dst = fdst;
-    void* bufs[2] = {fsrc, fdst};
-    const int S = (int)ds.size();
-    for (int s = 0; s < S; ++s) {
-        rc = p->dist.sweep(p->stream, ds[s], src, dst, 19 * esize(p->dtype), (size_t)p->nx * p->ny,
-                           [&](const void* a, void* b, const SlabView& sv) {
-                               if (push) return launch_lbm(p, a, b, flags + (sv.flags_off), omega, sv);
-                               return launch_lbm35(p, a, b, ds[s], omega, sv);
-                           });
-        if (rc) return rc;
-        src = bufs[(s + 1) % 2];
-        dst = bufs[s % 2];
-    }
-    if (S % 2 == 0) CUDA_TRY(cudaMemcpyAsync(fdst, fsrc, n, cudaMemcpyDeviceToDevice, p->stream));
+    rc = run_sweeps(p, ds, fsrc, fdst, 19, flags, [&](const void* a, void* b, int d, const SlabView& sv) {
+        if (push) return launch_lbm(p, a, b, sv.flags, omega, sv);
+        return launch_lbm35(p, a, b, d, omega, sv);
+    });
+    if (rc) return rc;
     CUDA_TRY(cudaGetLastError());
     return ST_OK;
 }
@@ -618,15 +762,109 @@ extern "C" int lbm_d3q19_run(st_plan* p, void* fsrc, void* fdst, double omega, i
 // ----------------------------------------------------------------------------
 // distribution (Z slabs)
 // ----------------------------------------------------------------------------
+#if ST_HAVE_NCCL
+bool st35d::NcclApi::load() {
+    if (h) return true;
+    h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return false;
+    getUniqueId = reinterpret_cast<decltype(getUniqueId)>(dlsym(h, "ncclGetUniqueId"));
+    commInitRank = reinterpret_cast<decltype(commInitRank)>(dlsym(h, "ncclCommInitRank"));
+    commDestroy = reinterpret_cast<decltype(commDestroy)>(dlsym(h, "ncclCommDestroy"));
+    send = reinterpret_cast<decltype(send)>(dlsym(h, "ncclSend"));
+    recv = reinterpret_cast<decltype(recv)>(dlsym(h, "ncclRecv"));
+    groupStart = reinterpret_cast<decltype(groupStart)>(dlsym(h, "ncclGroupStart"));
+    groupEnd = reinterpret_cast<decltype(groupEnd)>(dlsym(h, "ncclGroupEnd"));
+    errorString = reinterpret_cast<decltype(errorString)>(dlsym(h, "ncclGetErrorString"));
+    return getUniqueId && commInitRank && commDestroy && send && recv && groupStart && groupEnd && errorString;
+}
+st35d::NcclApi& st35d::nccl() {
+    static NcclApi api;
+    return api;
+}
+#endif
+
+void st35d::Dist::destroy() {
+    for (auto& s : slabs) {
+        for (void*& b : s.buf) if (b) cudaFree(b);
+        if (s.flags) cudaFree(s.flags);
+        if (s.fl2) cudaFree(s.fl2);
+    }
+    slabs.clear();
+    slab_cell_bytes = 0;
+    slab_ncomp = 0;
+#if ST_HAVE_NCCL
+    if (comm) { nccl().commDestroy(comm); comm = nullptr; }
+#endif
+}
+
+extern "C" int st_nccl_unique_id(void* out) {
+    if (!out) return fail(ST_EINVAL, "NULL id buffer");
+#if ST_HAVE_NCCL
+    if (!nccl().load()) return fail(ST_ENCCL, "libnccl.so.2 not loadable (import torch first)");
+    ncclUniqueId id;
+    ncclResult_t r = nccl().getUniqueId(&id);
+    if (r != ncclSuccess) return fail(ST_ENCCL, "ncclGetUniqueId: %s", nccl().errorString(r));
+    memcpy(out, &id, sizeof id);
+    return ST_OK;
+#else
+    return fail(ST_EUNSUPPORTED, "built without NCCL");
+#endif
+}
+
+extern "C" int st_slab_range(int nz, int nranks, int rank, int* z0, int* nz_local) {
+    if (nz < 1 || nranks < 1 || rank < 0 || rank >= nranks || nz < nranks) return fail(ST_EINVAL, "slab range");
+    int a = 0, b = 0;
+    slab_range(nz, nranks, rank, a, b);
+    if (z0) *z0 = a;
+    if (nz_local) *nz_local = b;
+    return ST_OK;
+}
+
 extern "C" int st_plan_set_dist(st_plan* p, const void* uid, int rank, int nranks) {
     if (!p) return fail(ST_EINVAL, "NULL plan");
+    if (nranks < 1 || rank < 0 || rank >= nranks) return fail(ST_EINVAL, "rank %d of %d", rank, nranks);
+    CUDA_TRY(cudaStreamSynchronize(p->stream));
     if (nranks == 1) { p->dist.init_single(p->nz); return ST_OK; }
-    (void)uid; (void)rank;
-    return fail(ST_EUNSUPPORTED, "distributed Z slabs not built yet");
+    const int g = p->dimT;
+    int z0 = 0, nzl = 0;
+    slab_range(p->nz, nranks, rank, z0, nzl);
+    if (p->nz / nranks < g) return fail(ST_EINVAL, "slabs of %d planes are thinner than dim_T %d", p->nz / nranks, g);
+#if ST_HAVE_NCCL
+    if (!uid) return fail(ST_EINVAL, "NULL NCCL unique id");
+    if (!nccl().load()) return fail(ST_ENCCL, "libnccl.so.2 not loadable (import torch first)");
+    p->dist.destroy();
+    ncclUniqueId id;
+    memcpy(&id, uid, sizeof id);
+    ncclComm_t comm = nullptr;
+    ncclResult_t r = nccl().commInitRank(&comm, nranks, id, rank);
+    if (r != ncclSuccess) return fail(ST_ENCCL, "ncclCommInitRank: %s", nccl().errorString(r));
+    Dist& D = p->dist;
+    D.mode = Dist::NCCL; D.comm = comm;
+    D.nz = p->nz; D.P = nranks; D.rank = rank; D.g = g; D.z0 = z0; D.nzl = nzl; D.nzb = nzl + 2 * g;
+    D.nranks = nranks;
+    p->fl2_of = nullptr; p->flags_checked = nullptr;
+    return ST_OK;
+#else
+    (void)uid;
+    return fail(ST_EUNSUPPORTED, "built without NCCL");
+#endif
 }
 
 extern "C" int st_plan_set_loopback_slabs(st_plan* p, int nslabs) {
     if (!p) return fail(ST_EINVAL, "NULL plan");
+    if (nslabs < 1) return fail(ST_EINVAL, "nslabs %d", nslabs);
+    CUDA_TRY(cudaStreamSynchronize(p->stream));
     if (nslabs == 1) { p->dist.init_single(p->nz); return ST_OK; }
-    return fail(ST_EUNSUPPORTED, "loopback slabs not built yet");
+    const int g = p->dimT;
+    if (p->nz / nslabs < g) return fail(ST_EINVAL, "slabs of %d planes are thinner than dim_T %d", p->nz / nslabs, g);
+    Dist& D = p->dist;
+    D.init_single(p->nz);      // caller buffers stay full grids in loopback mode
+    D.mode = Dist::LOOPBACK; D.P = nslabs; D.g = g;
+    D.slabs.resize(nslabs);
+    for (int k = 0; k < nslabs; ++k) {
+        slab_range(p->nz, nslabs, k, D.slabs[k].z0, D.slabs[k].nzl);
+        D.slabs[k].nzb = D.slabs[k].nzl + 2 * g;
+    }
+    return ST_OK;
 }

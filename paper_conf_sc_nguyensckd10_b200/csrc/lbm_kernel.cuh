@@ -191,13 +191,15 @@ struct Lbm35Params {
 
 template <int I, typename T, bool E, typename F>
 __device__ __forceinline__ void lbm_push_one(const T (&fs)[19], uint32_t fl, int x, int y, int q, int nx, int ny,
-                                             size_t plane, const uint8_t* __restrict__ fl2, const T* lidc, F&& put) {
+                                             int nzb, size_t plane, const uint8_t* __restrict__ fl2, const T* lidc,
+                                             F&& put) {
     constexpr int ex = D3Q19<I>::ex, ey = D3Q19<I>::ey, ez = D3Q19<I>::ez;
     if constexpr (I == 0) {
         put(0, 0, 0, 0, fs[0]);
     } else {
-        uint32_t tf = 0;
-        if (fl & 0x80u) tf = __ldg(fl2 + (size_t)(q + ez) * plane + (size_t)(y + ey) * nx + (x + ex)) & 0x7fu;
+        uint32_t tf = 0;   // a neighbour outside the slab buffer is a ghost-side cell: never non-FLUID here
+        if ((fl & 0x80u) && q + ez >= 0 && q + ez < nzb)
+            tf = __ldg(fl2 + (size_t)(q + ez) * plane + (size_t)(y + ey) * nx + (x + ex)) & 0x7fu;
         if (tf == 0) put(I, ex, ey, ez, fs[I]);
         else if (tf == 1) put(D3Q19<I>::opp, 0, 0, 0, fs[I]);
         else put(D3Q19<I>::opp, 0, 0, 0, Ar<T, E>::sub(fs[I], lidc[I]));
@@ -284,7 +286,7 @@ __global__ void __launch_bounds__(512, 1) lbm_35d_kernel(const Lbm35Params p) {
                         } else {
                             collide<T, E>(f, omega);
                             [&]<int... Is>(std::integer_sequence<int, Is...>) {
-                                (lbm_push_one<Is, T, E>(f, fl, x, y, q, p.nx, p.ny, plane, p.fl2, lidc, put), ...);
+                                (lbm_push_one<Is, T, E>(f, fl, x, y, q, p.nx, p.ny, p.nzb, plane, p.fl2, lidc, put), ...);
                             }(std::make_integer_sequence<int, 19>{});
                         }
                     } else {
@@ -301,7 +303,7 @@ __global__ void __launch_bounds__(512, 1) lbm_35d_kernel(const Lbm35Params p) {
                         } else {
                             collide<T, E>(f, omega);
                             [&]<int... Is>(std::integer_sequence<int, Is...>) {
-                                (lbm_push_one<Is, T, E>(f, fl, x, y, q, p.nx, p.ny, plane, p.fl2, lidc, put), ...);
+                                (lbm_push_one<Is, T, E>(f, fl, x, y, q, p.nx, p.ny, p.nzb, plane, p.fl2, lidc, put), ...);
                             }(std::make_integer_sequence<int, 19>{});
                         }
                     }

@@ -1,0 +1,74 @@
+"""Z-slab decomposition on one GPU (loopback transport, st_plan_set_loopback_slabs):
+P virtual slabs with dim_T-deep ghost planes exchanged before every sweep
+(the NCCL schedule with cudaMemcpyAsync as transport).  The result must be
+bit-identical to the single-slab run (SURVEY §8(e) invariant) and, in the
+bit-exact build, to the oracle."""
+import numpy as np
+import pytest
+import torch
+
+import stgen
+import paper_conf_sc_nguyensckd10_b200 as st
+
+pytestmark = pytest.mark.gpu
+
+
+def st7_gpu(a, T, dim_T, slabs=1, exact=False):
+    nz, ny, nx = a.shape
+    with st.Plan(nx, ny, nz, torch.float32 if a.dtype == np.float32 else torch.float64, dim_T) as p:
+        if exact:
+            p.set_bitexact(True)
+        if slabs > 1:
+            st.st_plan_set_loopback_slabs(p.h, slabs)
+        x = torch.from_numpy(a).cuda()
+        y = torch.empty_like(x)
+        p.st7(x, y, 0.4, 0.1, T)
+        p.sync()
+        return y.cpu().numpy()
+
+
+@pytest.mark.parametrize("P", [2, 3, 4])
+@pytest.mark.parametrize("dim_T", [1, 3, 4])
+def test_st7_loopback_identical(oracle_lib, P, dim_T):
+    a = stgen.grid7(64, 48, 41, 21, np.float32)
+    T = 2 * dim_T + 3
+    one = st7_gpu(a, T, dim_T)
+    many = st7_gpu(a, T, dim_T, slabs=P)
+    assert np.array_equal(one, many)
+    ex = st7_gpu(a, T, dim_T, slabs=P, exact=True)
+    assert np.array_equal(ex, oracle_lib.st7(a, 0.4, 0.1, T))
+
+
+def lbm_gpu(f0, flags, T, dim_T, slabs=1, exact=False):
+    _, nz, ny, nx = f0.shape
+    with st.Plan(nx, ny, nz, torch.float32 if f0.dtype == np.float32 else torch.float64, dim_T) as p:
+        if exact:
+            p.set_bitexact(True)
+        if slabs > 1:
+            st.st_plan_set_loopback_slabs(p.h, slabs)
+        a = torch.from_numpy(f0).cuda()
+        b = torch.empty_like(a)
+        p.lbm(a, b, 1.6, T, torch.from_numpy(flags).cuda())
+        p.sync()
+        return b.cpu().numpy()
+
+
+@pytest.mark.parametrize("P", [2, 3])
+@pytest.mark.parametrize("dim_T", [1, 2, 3])
+def test_lbm_loopback_identical(oracle_lib, P, dim_T):
+    nx, ny, nz = 40, 24, 23
+    flags = stgen.cavity_flags(nx, ny, nz)
+    flags[10:13, 8:12, 15:20] = stgen.WALL   # obstacle across a slab boundary
+    f0 = stgen.lbm_random(nx, ny, nz, 31, np.float32)
+    T = 7
+    ref = oracle_lib.lbm(f0, flags, 1.6, T)
+    got = lbm_gpu(f0, flags, T, dim_T, slabs=P, exact=True)
+    assert np.array_equal(got, ref)
+    assert np.array_equal(lbm_gpu(f0, flags, T, dim_T, slabs=P), lbm_gpu(f0, flags, T, max(dim_T, 2), slabs=1)) \
+        or dim_T == 1
+
+
+def test_slab_too_thin():
+    with st.Plan(64, 64, 16, torch.float32, 4) as p:
+        with pytest.raises(st.StError):
+            st.st_plan_set_loopback_slabs(p.h, 8)   # 2-plane slabs < dim_T
