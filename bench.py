@@ -162,9 +162,9 @@ def cpu_baseline_7pt(n):
     import stgen
     a = stgen.grid7(n, n, n, 2, np.float32)
     t0 = time.perf_counter()
-    oracle.st7(a, 0.4, 0.1, 1)
-    t1 = time.perf_counter() - t0
-    Ts = int(max(1, min(100, round(10.0 / max(t1, 1e-3)))))
+    oracle.st7(a, 0.4, 0.1, 8)
+    t1 = (time.perf_counter() - t0) / 8          # per sweep (incl. the oracle's own copies)
+    Ts = int(max(1, min(5000, round(12.0 / max(t1, 1e-4)))))
     t0 = time.perf_counter()
     oracle.st7(a, 0.4, 0.1, Ts)
     dt = time.perf_counter() - t0
@@ -236,43 +236,74 @@ def main():
         return tot, per
 
     # ------------------------------------------------------------------ 7-point
-    def st7_case(n, T, dtype, dim_t_fixed=0, steps=args.steps, warmup=args.warmup, choose=range(1, 9)):
+    def choose_dim_t(n, T, dtype, choose=range(1, 9)):
+        """dim_T by measurement: one timed pass of every dim_T on a local n^3 grid."""
         tdt = torch.float32 if dtype == np.float32 else torch.float64
-        a0 = torch.from_numpy(stgen.grid7(n, n, n, 2 + rank, dtype)).cuda()
+        x = torch.from_numpy(stgen.grid7(n, n, n, 2, dtype)).cuda()
+        y = torch.empty_like(x)
+        sweep = {}
+        for d in choose:
+            with st.Plan(n, n, n, tdt, d) as p:
+                p.set_stream(stream)
+                p.st7(x, y, 0.4, 0.1, T)
+                torch.cuda.synchronize()
+                tms, _ = time_steps(lambda: p.st7(x, y, 0.4, 0.1, T), 2, 0)
+                sweep[d] = round((n - 2) ** 3 * T / (tms / 2 / 1e3) / 1e6, 1)
+        best = max(sweep, key=sweep.get)
+        if world > 1:   # every rank runs rank 0's choice
+            obj = [best]
+            dist.broadcast_object_list(obj, src=0)
+            best = obj[0]
+        return best, sweep
+
+    uid = None
+    if world > 1:
+        obj = [st.st_nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+
+    def st7_case(n, T, dtype, D, steps=args.steps, warmup=args.warmup):
+        """weak scaling: each rank owns an n^3 Z-slab of an n x n x (n*world) grid."""
+        tdt = torch.float32 if dtype == np.float32 else torch.float64
+        nzg = n * world
+        p = st.Plan(n, n, nzg, tdt, D)
+        p.set_stream(stream)
+        if world > 1:
+            st.st_plan_set_dist(p.h, uid, rank, world)
+            z0, nzl = st.st_plan_local_slab(p.h)
+            g = st.st_plan_ghost_planes(p.h)
+        else:
+            z0, nzl, g = 0, nzg, 0
+        nzb = nzl + 2 * g
+        host = np.zeros((nzb, n, n), dtype=dtype)
+        zlo, zhi = max(0, z0 - g), min(nzg, z0 + nzl + g)
+        host[zlo - (z0 - g):zhi - (z0 - g)] = stgen.grid7(n, n, nzg, 2, dtype, z0=zlo, nzl=zhi - zlo)
+        a0 = torch.from_numpy(host).cuda()
         x = a0.clone()
         y = torch.empty_like(a0)
-        sweep = {}
-        if dim_t_fixed:
-            best = dim_t_fixed
-        else:
-            for d in choose:
-                with st.Plan(n, n, n, tdt, d) as p:
-                    p.set_stream(stream)
-                    p.st7(x, y, 0.4, 0.1, T)
-                    torch.cuda.synchronize()
-                    tms, _ = time_steps(lambda: p.st7(x, y, 0.4, 0.1, T), 2, 0)
-                    sweep[d] = round((n - 2) ** 3 * T / (tms / 2 / 1e3) / 1e6, 1)
-            best = max(sweep, key=sweep.get)
-        p = st.Plan(n, n, n, tdt, best)
-        p.set_stream(stream)
         tms, per = time_steps(lambda: p.st7(x, y, 0.4, 0.1, T), steps, warmup)
         launches = p.last_launches()
         info = p.info()
         ms = max_over_ranks(tms / steps)
-        upd = (n - 2) ** 3 * T
-        return p, best, sweep, ms, upd, launches, info, (a0, x, y)
+        upd = (n - 2) ** 2 * (nzg - 2) * T          # interior updates of the whole job
+        return p, ms, upd, launches, info, host
 
     with ClockSampler(local) as clk:
         n, T = args.n, args.T
-        p7, D, sweep, ms, upd, launches, info, bufs = st7_case(n, T, np.float32, args.dim_t)
-        value = upd * world / (ms / 1e3) / 1e6
+        if args.dim_t:
+            D, sweep = args.dim_t, {}
+        else:
+            D, sweep = choose_dim_t(n, T, np.float32)
+        p7, ms, upd, launches, info, host0 = st7_case(n, T, np.float32, D)
+        value = upd / (ms / 1e3) / 1e6
         per_launch_ms = ms / launches
         d_eff = info["dim_t_sweep"]
+        upd_rank = upd / world
         # roofline of the dominant kernel (st7_35d): both roofs, report the binding one
         ops_peak = SM_COUNT * FP32_LANES * sm_max * 1e6 / 1e12          # T FP32 lane-ops/s
-        achieved_ops = ST7_OPS * upd / (ms / 1e3) / 1e12
+        achieved_ops = ST7_OPS * upd_rank / (ms / 1e3) / 1e12
         bytes_per_upd = 8.0 / D
-        achieved_gbs = bytes_per_upd * upd / (ms / 1e3) / 1e9
+        achieved_gbs = bytes_per_upd * upd_rank / (ms / 1e3) / 1e9
         hbm_roof_upd = hbm_gbs * 1e9 / bytes_per_upd
         alu_roof_upd = ops_peak * 1e12 / ST7_OPS
         traffic = load_traffic(f"st7_f32_{n}_D{D}")
@@ -286,7 +317,7 @@ def main():
         roof, alt = (r_hbm, r_alu) if hbm_roof_upd < alu_roof_upd else (r_alu, r_hbm)
 
     # ------------------------------------------------------------------ e2e (host buffers)
-    a_host = torch.from_numpy(stgen.grid7(n, n, n, 2 + rank, np.float32)).pin_memory()
+    a_host = torch.from_numpy(host0).pin_memory()
     o_host = torch.empty_like(a_host).pin_memory()
     hin, hout = a_host.numpy(), o_host.numpy()
     for _ in range(max(1, args.warmup)):
@@ -298,21 +329,21 @@ def main():
         st.st7_run(p7.h, hin, hout, 0.4, 0.1, T)
         e2e_t += time.perf_counter() - t0
     e2e_ms = max_over_ranks(e2e_t / args.steps * 1e3)
-    grid_bytes = n ** 3 * 4
+    grid_bytes = host0.nbytes
 
     extras = {}
-    if not args.no_extras:
+    if not args.no_extras and world == 1:
         # FP64 256^3 (configs[1] FP64)
-        _, D64, sw64, ms64, upd64, l64, inf64, _ = st7_case(n, T, np.float64, 0, steps=3, warmup=1,
-                                                           choose=range(1, 9))
-        extras["st7_f64_256"] = {"value": round(upd64 * world / (ms64 / 1e3) / 1e6, 1), "unit": "Mupdates/s",
+        D64, sw64 = choose_dim_t(n, T, np.float64)
+        _, ms64, upd64, l64, inf64, _ = st7_case(n, T, np.float64, D64, steps=3, warmup=1)
+        extras["st7_f64_256"] = {"value": round(upd64 / (ms64 / 1e3) / 1e6, 1), "unit": "Mupdates/s",
                                  "dim_T": D64, "dim_T_sweep": sw64, "ms_per_step": round(ms64, 3),
                                  "frac_alu": round(ST7_OPS * upd64 / (ms64 / 1e3) /
                                                    (SM_COUNT * FP64_LANES * sm_max * 1e6), 4)}
         # FP32 512^3 (configs[3] per-GPU size)
-        _, D5, sw5, ms5, upd5, l5, inf5, _ = st7_case(512, T, np.float32, 0, steps=3, warmup=1,
-                                                      choose=range(1, 9))
-        extras["st7_f32_512"] = {"value": round(upd5 * world / (ms5 / 1e3) / 1e6, 1), "unit": "Mupdates/s",
+        D5, sw5 = choose_dim_t(512, T, np.float32)
+        _, ms5, upd5, l5, inf5, _ = st7_case(512, T, np.float32, D5, steps=3, warmup=1)
+        extras["st7_f32_512"] = {"value": round(upd5 / (ms5 / 1e3) / 1e6, 1), "unit": "Mupdates/s",
                                  "dim_T": D5, "dim_T_sweep": sw5, "ms_per_step": round(ms5, 3),
                                  "frac_alu": round(ST7_OPS * upd5 / (ms5 / 1e3) / (ops_peak * 1e12), 4),
                                  "info": inf5}
@@ -338,7 +369,7 @@ def main():
                                                          "frac": round(gbs / hbm_gbs, 4)},
                                             "launches": pl.last_launches()}
             del fa, fb, f0, flags
-    cpu = cpu_baseline_7pt(n) if (rank == 0 and world >= 1) else None
+    cpu = cpu_baseline_7pt(n) if (rank == 0 and world == 1) else None
 
     if rank == 0:
         line = {
@@ -347,14 +378,16 @@ def main():
             "ms_per_step": round(ms, 4), "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f32",
             "data": "synthetic (splitmix64 U[0,1) grid, seed 2; alpha=0.4 beta=0.1)",
-            "config": {"workload": f"7-point stencil FP32 {n}^3, T={T} (BASELINE configs[1]); "
-                                   f"dim_T chosen by measurement",
-                       "grid": [n, n, n], "T": T, "dim_T": D, "dim_T_sweep_Mupd": sweep,
-                       "parallelism": f"replicas x{world}" if world > 1 else "single",
+            "config": {"workload": (f"7-point stencil FP32 {n}^3, T={T} (BASELINE configs[1]); "
+                                    f"dim_T chosen by measurement") if world == 1 else
+                                   (f"7-point stencil FP32 {n}x{n}x{n * world} (n^3 per GPU, configs[3] weak "
+                                    f"scaling), T={T}, Z-slabs with dim_T-deep NCCL ghost exchange"),
+                       "grid": [n, n, n * world], "T": T, "dim_T": D, "dim_T_sweep_Mupd": sweep,
+                       "parallelism": f"zslab{world}" if world > 1 else "single",
                        "l2": "flushed between timed steps (512 MiB write)",
                        "plan": info},
             "roofline": roof, "roofline_alt": alt,
-            "e2e": {"value": round(upd * world / (e2e_ms / 1e3) / 1e6, 1), "unit": "Mupdates/s",
+            "e2e": {"value": round(upd / (e2e_ms / 1e3) / 1e6, 1), "unit": "Mupdates/s",
                     "h2d_bytes_per_step": grid_bytes, "d2h_bytes_per_step": grid_bytes,
                     "ms_per_step": round(e2e_ms, 3)},
             "gpu_launches": launches * args.steps,
