@@ -173,10 +173,10 @@ static int plan7(st_plan* p, int d, int nzo, Geo7& g) {
         // TMA ring: as deep as shared memory allows (prefetch ring-2 planes ahead:
         // the plane loads must cover HBM latency, several rounds of compute)
         c.ring = 0;
-        for (int r = ST7_RING_MAX; r >= 4; --r)
+        for (int r = ST7_RING_MAX; r >= 5; --r)
             if (smem7(c, p->dtype, r) <= p->smem_optin) { c.ring = r; break; }
         if (const char* e = getenv("ST_RING")) c.ring = std::min(c.ring, atoi(e));
-        if (c.ring < 4) continue;
+        if (c.ring < 5) continue;
         c.smem = smem7(c, p->dtype, c.ring);
         long cost = (long)c.tiles_y * c.TY;
         if (best < 0 || cost < best || (cost == best && c.TY > g.TY)) {

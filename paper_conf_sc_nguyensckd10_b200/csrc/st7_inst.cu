@@ -62,6 +62,7 @@ St7LaunchFn ST_FN(int D, int VY, int MAXT) {
     if (VY == 4 && MAXT == 256) return pick<4, 256>(D);
     if (VY == 2 && MAXT == 256) return pick<2, 256>(D);
     if (VY == 2 && MAXT == 512) return pick<2, 512>(D);
+    if (VY == 4 && MAXT == 384) return pick<4, 384>(D);
     return nullptr;
 }
 

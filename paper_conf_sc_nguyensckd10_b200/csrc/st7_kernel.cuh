@@ -66,17 +66,17 @@ template <> struct Row<float> { float2 a, b; };
 template <> struct Row<double> { double v[2]; };
 
 template <int VY> struct Blk<float, VY> {
-    float2 a[VY], b[VY];
+    float2 a[VY], b[VY];   // natural pairs: a = (c0, c1), b = (c2, c3): 16-byte rows load/store with no moves
     __device__ __forceinline__ void load_nat(int j, const float* s) {   // smem, natural order
         const float4 v = *reinterpret_cast<const float4*>(s);
-        a[j] = make_float2(v.x, v.z);
-        b[j] = make_float2(v.y, v.w);
+        a[j] = make_float2(v.x, v.y);
+        b[j] = make_float2(v.z, v.w);
     }
-    __device__ __forceinline__ void store_x(int j, float4* s) const {   // exchange row, pair order
+    __device__ __forceinline__ void store_x(int j, float4* s) const {   // exchange row
         *s = make_float4(a[j].x, a[j].y, b[j].x, b[j].y);
     }
     __device__ __forceinline__ void store_global(int j, float* g) const {  // plain store: predicable
-        *reinterpret_cast<float4*>(g) = make_float4(a[j].x, b[j].x, a[j].y, b[j].y);
+        *reinterpret_cast<float4*>(g) = make_float4(a[j].x, a[j].y, b[j].x, b[j].y);
     }
 };
 template <int VY> struct Blk<double, VY> {
@@ -93,7 +93,7 @@ template <int VY> struct Blk<double, VY> {
 
 __device__ __forceinline__ Row<float> row_nat(const float* s) {
     const float4 v = *reinterpret_cast<const float4*>(s);
-    return Row<float>{make_float2(v.x, v.z), make_float2(v.y, v.w)};
+    return Row<float>{make_float2(v.x, v.y), make_float2(v.z, v.w)};
 }
 __device__ __forceinline__ Row<float> row_x(const float4* s) {
     const float4 v = *s;
@@ -123,16 +123,16 @@ __device__ __forceinline__ float2 combine_exact(float al, float2 c, float be, fl
 // warp-uniform branch; whole z-shell planes use Coef::fixed().
 template <typename T> struct Coef;
 template <> struct Coef<float> {
-    float2 alA, beA, alB, beB;     // for the pairs a = (c0, c2), b = (c1, c3)
+    float2 alA, beA, alB, beB;     // for the pairs a = (c0, c1), b = (c2, c3)
     static __device__ __forceinline__ Coef fixed() {
         return Coef{make_float2(1.f, 1.f), make_float2(0.f, 0.f), make_float2(1.f, 1.f), make_float2(0.f, 0.f)};
     }
     static __device__ __forceinline__ Coef make(float al, float be, uint32_t xfix) {  // xfix bit i: column i fixed
         Coef k;
-        k.alA = make_float2(xfix & 1 ? 1.f : al, xfix & 4 ? 1.f : al);
-        k.beA = make_float2(xfix & 1 ? 0.f : be, xfix & 4 ? 0.f : be);
-        k.alB = make_float2(xfix & 2 ? 1.f : al, xfix & 8 ? 1.f : al);
-        k.beB = make_float2(xfix & 2 ? 0.f : be, xfix & 8 ? 0.f : be);
+        k.alA = make_float2(xfix & 1 ? 1.f : al, xfix & 2 ? 1.f : al);
+        k.beA = make_float2(xfix & 1 ? 0.f : be, xfix & 2 ? 0.f : be);
+        k.alB = make_float2(xfix & 4 ? 1.f : al, xfix & 8 ? 1.f : al);
+        k.beB = make_float2(xfix & 4 ? 0.f : be, xfix & 8 ? 0.f : be);
         return k;
     }
 };
@@ -156,10 +156,18 @@ __device__ __forceinline__ void st7_level(const Blk<float, VY>& ZM, const Blk<fl
         const float right = __shfl_down_sync(0xffffffffu, C.a[j].x, 1, NTX);  // x0 + 4
         const float2 yma = j > 0 ? C.a[j - 1] : top.a, ypa = j < VY - 1 ? C.a[j + 1] : bot.a;
         const float2 ymb = j > 0 ? C.b[j - 1] : top.b, ypb = j < VY - 1 ? C.b[j + 1] : bot.b;
-        const float2 sxa = __fadd2_rn(make_float2(left, C.b[j].x), C.b[j]);
-        const float2 sxb = __fadd2_rn(C.a[j], make_float2(C.a[j].y, right));
-        const float2 sa = __fadd2_rn(__fadd2_rn(sxa, __fadd2_rn(yma, ypa)), __fadd2_rn(ZM.a[j], ZP.a[j]));
-        const float2 sb = __fadd2_rn(__fadd2_rn(sxb, __fadd2_rn(ymb, ypb)), __fadd2_rn(ZM.b[j], ZP.b[j]));
+        // X sums: (x-1 + x+1) for (c0, c1) = (L, c0) + (c1, c2); for (c2, c3) = (c1, c2) + (c3, R)
+        const float2 mid = make_float2(C.a[j].y, C.b[j].x);
+        const float2 sxa = __fadd2_rn(make_float2(left, C.a[j].x), mid);
+        const float2 sxb = __fadd2_rn(mid, make_float2(C.b[j].y, right));
+        float2 sa, sb;
+        if (EXACT) {   // oracle order (X2)
+            sa = __fadd2_rn(__fadd2_rn(sxa, __fadd2_rn(yma, ypa)), __fadd2_rn(ZM.a[j], ZP.a[j]));
+            sb = __fadd2_rn(__fadd2_rn(sxb, __fadd2_rn(ymb, ypb)), __fadd2_rn(ZM.b[j], ZP.b[j]));
+        } else {       // shuffled X terms last: the y/z sums overlap the shuffle latency
+            sa = __fadd2_rn(__fadd2_rn(__fadd2_rn(yma, ypa), __fadd2_rn(ZM.a[j], ZP.a[j])), sxa);
+            sb = __fadd2_rn(__fadd2_rn(__fadd2_rn(ymb, ypb), __fadd2_rn(ZM.b[j], ZP.b[j])), sxb);
+        }
         if (EXACT) {
             R.a[j] = make_float2(__fadd_rn(__fmul_rn(k.alA.x, C.a[j].x), __fmul_rn(k.beA.x, sa.x)),
                                  __fadd_rn(__fmul_rn(k.alA.y, C.a[j].y), __fmul_rn(k.beA.y, sa.y)));
@@ -220,13 +228,17 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
     const int TY = NTY * VY;
     const T al = T(p.alpha), be = T(p.beta);
 
-    const int RING = p.ring, PF = p.ring - 2;
+    const int RING = p.ring, PF = p.ring - 3;   // ring keeps planes r-2, r-1, r for level 1
     T* ring = reinterpret_cast<T*>(smem_raw);                      // [RING][TY][TX]
     const int slot_elems = TX * TY;
     // row exchange buffer [level 1..D-1][parity][N row / S row][MAXT] (16-byte rows)
     V* xbuf = reinterpret_cast<V*>(ring + RING * slot_elems);
     uint64_t* bars = reinterpret_cast<uint64_t*>(xbuf + (D > 1 ? (D - 1) * 4 * MAXT : 0));
 
+    // zero the ring once: a boundary plane is formed as 1*c + 0*s and may read a
+    // never-loaded neighbour plane slot, which must hold finite values
+    for (int i = tid; i < RING * slot_elems; i += blockDim.x) ring[i] = T(0);
+    fence_proxy_async();   // generic-proxy writes before the first TMA (async proxy) writes
     if (tid == 0) {
         prefetch_tensormap(&tmap);
         for (int s = 0; s < RING; ++s) mbar_init(&bars[s], 1);
@@ -234,11 +246,12 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
     }
     __syncthreads();
 
-    // register planes: level l (0..D-1), rotating slot (prev / cur / new)
+    // register planes: level l (1..D-1), rotating slot (prev / cur / new); level 0
+    // is read straight from the TMA ring (index 0 unused)
     B pl[D][3];
     B outv;
 #pragma unroll
-    for (int l = 0; l < D; ++l)
+    for (int l = 1; l < D; ++l)
 #pragma unroll
         for (int k = 0; k < 3; ++k) pl[l][k] = B{};   // finite (see Coef)
 
@@ -312,6 +325,7 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
         uint32_t slot_r = kbase % RING, par_r = (kbase / RING) & 1;       // for plane r
         uint32_t slot_f = (kbase + PF) % RING;                            // for plane r + PF
         uint32_t slot_m1 = (slot_r + RING - 1) % RING;                    // for plane r - 1
+        uint32_t slot_m2 = (slot_r + RING - 2) % RING;                    // for plane r - 2
         // output row pointer of plane r - D (level D at round r), advanced by one plane per round
         T* pout = outcol + (long long)(r0 - D) * (long long)plane;
         const int nxs = p.nx;
@@ -326,13 +340,8 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                 mbar_arrive_expect_tx(bar, tile_bytes);
                 tma_load_3d(ring + slot_f * slot_elems, &tmap, bar, Lx, Ly, r + PF);
             }
-            // level 0: plane r from the ring into registers
-            if (STEADY || r <= rl1) {
-                mbar_wait(&bars[slot_r], par_r);
-                const T* sl = ring + slot_r * slot_elems + my_off;
-#pragma unroll
-                for (int j = 0; j < VY; ++j) pl[0][NEW].load_nat(j, sl + j * TX);
-            }
+            // level 0: plane r has landed in the ring
+            if (STEADY || r <= rl1) mbar_wait(&bars[slot_r], par_r);
             const int rpar = r & 1;
             // levels 1..D: level l computes plane z = r - l
 #pragma unroll
@@ -356,13 +365,31 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                     top = row_x(xtop + o);
                     bot = row_x(xbot + o);
                 }
-                B& dst = l < D ? pl[l < D ? l : 0][NEW] : outv;
-                if (!STEADY && zfix)
-                    st7_level<NTX, VY, EXACT>(pl[l - 1][PREV], pl[l - 1][CUR], pl[l - 1][NEW], top, bot,
-                                              Coef<T>::fixed(), yslow, rowfix, dst);
-                else
-                    st7_level<NTX, VY, EXACT>(pl[l - 1][PREV], pl[l - 1][CUR], pl[l - 1][NEW], top, bot, kc,
-                                              yslow, rowfix, dst);
+                B& dst = l < D ? pl[l < D ? l : 1][NEW] : outv;
+                if (l == 1) {   // level-0 planes r-2, r-1, r of my block straight from the ring
+                    B zm, c, zp;
+                    const T* s2 = ring + slot_m2 * slot_elems + my_off;
+                    const T* s1 = ring + slot_m1 * slot_elems + my_off;
+                    const T* s0 = ring + slot_r * slot_elems + my_off;
+#pragma unroll
+                    for (int j = 0; j < VY; ++j) {
+                        zm.load_nat(j, s2 + j * TX);
+                        c.load_nat(j, s1 + j * TX);
+                        zp.load_nat(j, s0 + j * TX);
+                    }
+                    if (!STEADY && zfix)
+                        st7_level<NTX, VY, EXACT>(zm, c, zp, top, bot, Coef<T>::fixed(), yslow, rowfix, dst);
+                    else
+                        st7_level<NTX, VY, EXACT>(zm, c, zp, top, bot, kc, yslow, rowfix, dst);
+                } else {
+                    const int lp = l > 1 ? l - 1 : 1;
+                    if (!STEADY && zfix)
+                        st7_level<NTX, VY, EXACT>(pl[lp][PREV], pl[lp][CUR], pl[lp][NEW], top, bot,
+                                                  Coef<T>::fixed(), yslow, rowfix, dst);
+                    else
+                        st7_level<NTX, VY, EXACT>(pl[lp][PREV], pl[lp][CUR], pl[lp][NEW], top, bot, kc,
+                                                  yslow, rowfix, dst);
+                }
                 if (l < D) {
                     V* xb = xw + ((l - 1) * 4 + zpar * 2) * MAXT;
                     dst.store_x(0, xb);
@@ -376,6 +403,7 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
             __syncthreads();
             pout += plane;
             // advance the ring cursors
+            slot_m2 = slot_m1;
             slot_m1 = slot_r;
             if (++slot_r == (uint32_t)RING) { slot_r = 0; par_r ^= 1; }
             if (++slot_f == (uint32_t)RING) slot_f = 0;
