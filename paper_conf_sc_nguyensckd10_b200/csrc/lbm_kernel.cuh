@@ -87,14 +87,24 @@ __device__ __forceinline__ T edotu(T ux, T uy, T uz) {
 template <typename T, bool E>
 __device__ __forceinline__ void collide(T (&f)[19], T omega) {
     using A = Ar<T, E>;
-    T rho = f[0];
+    T rho, jx, jy, jz;
+    if (E) {   // oracle order (X20): sequential sums in index order
+        rho = f[0];
 #pragma unroll
-    for (int i = 1; i < 19; ++i) rho = A::add(rho, f[i]);
-    T jx, jy, jz;
-    bool fx = true, fy = true, fz = true;
-    jsum<T, E, 0>(f, jx, fx);
-    jsum<T, E, 1>(f, jy, fy);
-    jsum<T, E, 2>(f, jz, fz);
+        for (int i = 1; i < 19; ++i) rho = A::add(rho, f[i]);
+        bool fx = true, fy = true, fz = true;
+        jsum<T, E, 0>(f, jx, fx);
+        jsum<T, E, 1>(f, jy, fy);
+        jsum<T, E, 2>(f, jz, fz);
+    } else {   // tolerance mode (X20): tree-ordered sums, depth 5 instead of 18
+        const T s01 = f[1] + f[2], s34 = f[3] + f[4], s56 = f[5] + f[6];
+        const T s78 = f[7] + f[8], s910 = f[9] + f[10], s1112 = f[11] + f[12], s1314 = f[13] + f[14];
+        const T s1516 = f[15] + f[16], s1718 = f[17] + f[18];
+        rho = ((f[0] + (s01 + s34)) + (s56 + s78)) + ((s910 + s1112) + (s1314 + (s1516 + s1718)));
+        jx = ((f[1] - f[2]) + (f[7] - f[8])) + ((f[9] - f[10]) + ((f[11] - f[12]) + (f[13] - f[14])));
+        jy = ((f[3] - f[4]) + (f[7] - f[8])) + ((f[10] - f[9]) + ((f[15] - f[16]) + (f[17] - f[18])));
+        jz = ((f[5] - f[6]) + (f[11] - f[12])) + ((f[14] - f[13]) + ((f[15] - f[16]) + (f[18] - f[17])));
+    }
     const T ux = A::div(jx, rho), uy = A::div(jy, rho), uz = A::div(jz, rho);
     T usq = A::add(A::mul(ux, ux), A::mul(uy, uy));
     usq = A::add(usq, A::mul(uz, uz));
