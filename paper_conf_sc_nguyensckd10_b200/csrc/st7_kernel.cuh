@@ -346,6 +346,7 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
             // levels 1..D: level l computes plane z = r - l
 #pragma unroll
             for (int l = 1; l <= D; ++l) {
+                if (p.dbg & 1) break;   // tuning only: stream the planes without computing
                 const int z = r - l;
                 bool zfix = false;
                 if (!STEADY) {
