@@ -381,7 +381,8 @@ static int launch7(st_plan* p, const void* src, void* dst, int d, double alpha, 
     if (const char* e = getenv("ST_DBG")) prm.dbg = atoi(e);
     prm.alpha = alpha; prm.beta = beta;
     if (prm.work <= 0) return ST_OK;
-    cudaError_t e = g->fn(&map, prm, g->grid, g->threads, g->smem, sv.stream ? sv.stream : p->stream);
+    const int grid = sv.grid_cap > 0 ? std::min(g->grid, sv.grid_cap) : g->grid;
+    cudaError_t e = g->fn(&map, prm, grid, g->threads, g->smem, sv.stream ? sv.stream : p->stream);
     if (e != cudaSuccess) return fail(ST_ECUDA, "st7 launch (d=%d): %s", d, cudaGetErrorString(e));
     ++p->launches;
     return ST_OK;
@@ -392,7 +393,7 @@ static int launch7(st_plan* p, const void* src, void* dst, int d, double alpha, 
 // ----------------------------------------------------------------------------
 // ncomp: SoA components of a cell (1 for the 7-point grid, 19 for D3Q19); each
 // component of a slab buffer is nzb consecutive planes.
-static int exchange_nccl(st_plan* p, void* buf, int d, int ncomp) {
+static int exchange_nccl(st_plan* p, void* buf, int d, int ncomp, cudaStream_t st) {
 #if ST_HAVE_NCCL
     Dist& D = p->dist;
     const size_t pb = (size_t)p->nx * p->ny * esize(p->dtype);
@@ -404,12 +405,12 @@ static int exchange_nccl(st_plan* p, void* buf, int d, int ncomp) {
     for (int c = 0; c < ncomp && r == ncclSuccess; ++c) {
         char* base = b + c * cs;
         if (D.rank > 0) {
-            if (r == ncclSuccess) r = N.send(base + (size_t)D.g * pb, bytes, ncclUint8, D.rank - 1, D.comm, p->stream);
-            if (r == ncclSuccess) r = N.recv(base + (size_t)(D.g - d) * pb, bytes, ncclUint8, D.rank - 1, D.comm, p->stream);
+            if (r == ncclSuccess) r = N.send(base + (size_t)D.g * pb, bytes, ncclUint8, D.rank - 1, D.nccl_comm, st);
+            if (r == ncclSuccess) r = N.recv(base + (size_t)(D.g - d) * pb, bytes, ncclUint8, D.rank - 1, D.nccl_comm, st);
         }
         if (D.rank < D.P - 1) {
-            if (r == ncclSuccess) r = N.send(base + (size_t)(D.g + D.nzl - d) * pb, bytes, ncclUint8, D.rank + 1, D.comm, p->stream);
-            if (r == ncclSuccess) r = N.recv(base + (size_t)(D.g + D.nzl) * pb, bytes, ncclUint8, D.rank + 1, D.comm, p->stream);
+            if (r == ncclSuccess) r = N.send(base + (size_t)(D.g + D.nzl - d) * pb, bytes, ncclUint8, D.rank + 1, D.nccl_comm, st);
+            if (r == ncclSuccess) r = N.recv(base + (size_t)(D.g + D.nzl) * pb, bytes, ncclUint8, D.rank + 1, D.nccl_comm, st);
         }
     }
     ncclResult_t r2 = N.groupEnd();
@@ -417,12 +418,12 @@ static int exchange_nccl(st_plan* p, void* buf, int d, int ncomp) {
         return fail(ST_ENCCL, "ghost exchange: %s", N.errorString(r != ncclSuccess ? r : r2));
     return ST_OK;
 #else
-    (void)p; (void)buf; (void)d; (void)ncomp;
+    (void)p; (void)buf; (void)d; (void)ncomp; (void)st;
     return fail(ST_EUNSUPPORTED, "built without NCCL");
 #endif
 }
 
-static int exchange_loop(st_plan* p, int cur, int d, int ncomp) {
+static int exchange_loop(st_plan* p, int cur, int d, int ncomp, cudaStream_t st) {
     Dist& D = p->dist;
     const size_t pb = (size_t)p->nx * p->ny * esize(p->dtype);
     const size_t bytes = (size_t)d * pb;
@@ -437,7 +438,7 @@ static int exchange_loop(st_plan* p, int cur, int d, int ncomp) {
             for (int c = 0; c < ncomp; ++c)
                 CUDA_TRY(cudaMemcpyAsync(me + c * cs + (size_t)(D.g - d) * pb,
                                          src + c * ocs + (size_t)(D.g + o.nzl - d) * pb, bytes,
-                                         cudaMemcpyDeviceToDevice, p->stream));
+                                         cudaMemcpyDeviceToDevice, st));
         }
         if (k < D.P - 1) {
             Dist::Slab& o = D.slabs[k + 1];
@@ -445,7 +446,7 @@ static int exchange_loop(st_plan* p, int cur, int d, int ncomp) {
             const size_t ocs = (size_t)o.nzb * pb;
             for (int c = 0; c < ncomp; ++c)
                 CUDA_TRY(cudaMemcpyAsync(me + c * cs + (size_t)(D.g + s.nzl) * pb, src + c * ocs + (size_t)D.g * pb,
-                                         bytes, cudaMemcpyDeviceToDevice, p->stream));
+                                         bytes, cudaMemcpyDeviceToDevice, st));
         }
     }
     return ST_OK;
@@ -493,60 +494,114 @@ static int ensure_loop_slabs(st_plan* p, int ncomp, const uint8_t* flags) {
     return ST_OK;
 }
 
+static int ensure_comm(st_plan* p) {
+    Dist& D = p->dist;
+    if (!D.comm) CUDA_TRY(cudaStreamCreateWithFlags(&D.comm, cudaStreamNonBlocking));
+    if (!D.ev_b) CUDA_TRY(cudaEventCreateWithFlags(&D.ev_b, cudaEventDisableTiming));
+    if (!D.ev_x) CUDA_TRY(cudaEventCreateWithFlags(&D.ev_x, cudaEventDisableTiming));
+    return ST_OK;
+}
+
+// Sweeps over Z slabs with the ghost exchange for sweep k+1 overlapped with
+// the interior of sweep k: the d' output planes next to each
+// slab face are computed first, an event hands them to the exchange stream,
+// the interior planes are computed meanwhile, and sweep k+1 waits for the
+// exchange.  ST_NO_OVERLAP=1 serialises exchange and sweep (A/B tuning).
 template <typename L>
 static int run_sweeps(st_plan* p, const std::vector<int>& ds, const void* in, void* out, int ncomp,
                       const uint8_t* flags, L&& launch) {
     Dist& D = p->dist;
     const size_t pb = (size_t)p->nx * p->ny * esize(p->dtype);
-    if (D.mode == Dist::LOOPBACK) {
-        int rc = ensure_loop_slabs(p, ncomp, flags);
+    const bool overlap_ok = getenv("ST_NO_OVERLAP") == nullptr;
+    if (D.mode == Dist::SINGLE) {
+        const void* src = in;
+        void* dst = out;
+        void* bufs[2] = {const_cast<void*>(in), out};
+        for (size_t k = 0; k < ds.size(); ++k) {
+            SlabView sv;
+            sv.stream = p->stream; sv.flags = flags; sv.fl2 = p->fl2;
+            sv.nzb = p->nz; sv.zbase = 0; sv.za = 0; sv.zb = p->nz; sv.single = true;
+            int rc = launch(src, dst, ds[k], sv);
+            if (rc) return rc;
+            src = bufs[(k + 1) % 2];
+            dst = bufs[k % 2];
+        }
+        if (ds.size() % 2 == 0)  // only when every sweep has depth 1 and T is even: result in `in`
+            CUDA_TRY(cudaMemcpyAsync(out, in, (size_t)ncomp * D.nzb * pb, cudaMemcpyDeviceToDevice, p->stream));
+        return ST_OK;
+    }
+    int rc = ensure_comm(p);
+    if (rc) return rc;
+    const bool loop = D.mode == Dist::LOOPBACK;
+    // slab list: loopback = every virtual slab; NCCL = this rank's slab in the caller's buffers
+    struct S { void* buf[2]; int z0, nzl, nzb; const uint8_t* flags; uint8_t* fl2; };
+    std::vector<S> sl;
+    if (loop) {
+        rc = ensure_loop_slabs(p, ncomp, flags);
         if (rc) return rc;
         for (auto& s : D.slabs) {   // scatter owned planes + available ghosts
             const int zlo = std::max(0, s.z0 - D.g), zhi = std::min(p->nz, s.z0 + s.nzl + D.g);
             rc = slab_copy(p, const_cast<void*>(in), s.buf[0], s.z0 - D.g, s.nzb, zlo, zhi - zlo, ncomp, true);
             if (rc) return rc;
+            sl.push_back({{s.buf[0], s.buf[1]}, s.z0, s.nzl, s.nzb, s.flags, s.fl2});
         }
-        int cur = 0;
-        for (size_t k = 0; k < ds.size(); ++k) {
-            rc = exchange_loop(p, cur, ds[k], ncomp);
-            if (rc) return rc;
-            for (auto& s : D.slabs) {
-                SlabView sv;
-                sv.nzb = s.nzb; sv.zbase = s.z0 - D.g; sv.za = D.g; sv.zb = D.g + s.nzl;
-                sv.flags = s.flags; sv.fl2 = s.fl2; sv.single = false; sv.stream = p->stream;
-                rc = launch(s.buf[cur], s.buf[1 - cur], ds[k], sv);
+    } else {
+        sl.push_back({{const_cast<void*>(in), out}, D.z0, D.nzl, D.nzb, flags, p->fl2});
+    }
+    auto exchange = [&](int which, int d, cudaStream_t st) -> int {
+        if (loop) return exchange_loop(p, which, d, ncomp, st);
+        return exchange_nccl(p, sl[0].buf[which], d, ncomp, st);
+    };
+    auto view = [&](const S& s, int za, int zb, int cap) {
+        SlabView sv;
+        sv.nzb = s.nzb; sv.zbase = s.z0 - D.g; sv.za = za; sv.zb = zb;
+        sv.flags = s.flags; sv.fl2 = s.fl2; sv.single = false; sv.stream = p->stream; sv.grid_cap = cap;
+        return sv;
+    };
+    int cur = 0;
+    rc = exchange(cur, ds[0], p->stream);   // ghosts of the input
+    if (rc) return rc;
+    const int cap = loop ? 0 : std::max(1, p->sms - 8);   // leave SMs to the NCCL kernels
+    for (size_t k = 0; k < ds.size(); ++k) {
+        const int d = ds[k], dn = k + 1 < ds.size() ? ds[k + 1] : 0;
+        bool split = overlap_ok && dn > 0;
+        for (auto& s : sl) split = split && s.nzl > 2 * dn;
+        if (split) {
+            for (auto& s : sl) {   // boundary planes first
+                rc = launch(s.buf[cur], s.buf[1 - cur], d, view(s, D.g, D.g + dn, 0));
+                if (!rc) rc = launch(s.buf[cur], s.buf[1 - cur], d, view(s, D.g + s.nzl - dn, D.g + s.nzl, 0));
                 if (rc) return rc;
             }
-            cur ^= 1;
-        }
-        for (auto& s : D.slabs) {   // gather owned planes
-            rc = slab_copy(p, out, s.buf[cur], s.z0 - D.g, s.nzb, s.z0, s.nzl, ncomp, false);
+            CUDA_TRY(cudaEventRecord(D.ev_b, p->stream));
+            CUDA_TRY(cudaStreamWaitEvent(D.comm, D.ev_b, 0));
+            rc = exchange(1 - cur, dn, D.comm);
             if (rc) return rc;
-        }
-        return ST_OK;
-    }
-    const void* src = in;
-    void* dst = out;
-    void* bufs[2] = {const_cast<void*>(in), out};
-    for (size_t k = 0; k < ds.size(); ++k) {
-        SlabView sv;
-        sv.stream = p->stream;
-        sv.flags = flags;
-        sv.fl2 = p->fl2;
-        if (D.mode == Dist::NCCL) {
-            int rc = exchange_nccl(p, const_cast<void*>(src), ds[k], ncomp);
-            if (rc) return rc;
-            sv.nzb = D.nzb; sv.zbase = D.z0 - D.g; sv.za = D.g; sv.zb = D.g + D.nzl; sv.single = false;
+            CUDA_TRY(cudaEventRecord(D.ev_x, D.comm));
+            for (auto& s : sl) {   // interior overlaps the exchange
+                rc = launch(s.buf[cur], s.buf[1 - cur], d, view(s, D.g + dn, D.g + s.nzl - dn, cap));
+                if (rc) return rc;
+            }
+            CUDA_TRY(cudaStreamWaitEvent(p->stream, D.ev_x, 0));
         } else {
-            sv.nzb = p->nz; sv.zbase = 0; sv.za = 0; sv.zb = p->nz; sv.single = true;
+            for (auto& s : sl) {
+                rc = launch(s.buf[cur], s.buf[1 - cur], d, view(s, D.g, D.g + s.nzl, 0));
+                if (rc) return rc;
+            }
+            if (dn > 0) {
+                rc = exchange(1 - cur, dn, p->stream);
+                if (rc) return rc;
+            }
         }
-        int rc = launch(src, dst, ds[k], sv);
-        if (rc) return rc;
-        src = bufs[(k + 1) % 2];
-        dst = bufs[k % 2];
+        cur ^= 1;
     }
-    if (ds.size() % 2 == 0)  // only when every sweep has depth 1 and T is even: result in `in`
+    if (loop) {
+        for (auto& s : D.slabs) {   // gather owned planes
+            rc = slab_copy(p, out, cur == 0 ? s.buf[0] : s.buf[1], s.z0 - D.g, s.nzb, s.z0, s.nzl, ncomp, false);
+            if (rc) return rc;
+        }
+    } else if (cur == 0) {   // even number of sweeps: the result is in `in`
         CUDA_TRY(cudaMemcpyAsync(out, in, (size_t)ncomp * D.nzb * pb, cudaMemcpyDeviceToDevice, p->stream));
+    }
     return ST_OK;
 }
 
@@ -652,7 +707,8 @@ static int launch_lbm35(st_plan* p, const void* src, void* dst, int d, double om
     if (p->dtype == ST_F32) lid_coeffs<float>(p->lid, prm.lidc);
     else lid_coeffs<double>(p->lid, prm.lidc);
     if (prm.work <= 0) return ST_OK;
-    const int grid = (int)std::min<long long>(p->sms, prm.work);
+    int grid = (int)std::min<long long>(p->sms, prm.work);
+    if (sv.grid_cap > 0) grid = std::min(grid, sv.grid_cap);
     cudaError_t e = lbm35_launch(p->dtype == ST_F32 ? 0 : 1, p->exact, d, prm, grid, 32 * g.TY, g.smem,
                                  sv.stream ? sv.stream : p->stream);
     if (e != cudaSuccess) return fail(ST_ECUDA, "lbm_35d launch (d=%d): %s", d, cudaGetErrorString(e));
@@ -794,8 +850,11 @@ void st35d::Dist::destroy() {
     slab_cell_bytes = 0;
     slab_ncomp = 0;
 #if ST_HAVE_NCCL
-    if (comm) { nccl().commDestroy(comm); comm = nullptr; }
+    if (nccl_comm) { nccl().commDestroy(nccl_comm); nccl_comm = nullptr; }
 #endif
+    if (comm) { cudaStreamSynchronize(comm); cudaStreamDestroy(comm); comm = nullptr; }
+    if (ev_b) { cudaEventDestroy(ev_b); ev_b = nullptr; }
+    if (ev_x) { cudaEventDestroy(ev_x); ev_x = nullptr; }
 }
 
 extern "C" int st_nccl_unique_id(void* out) {
@@ -840,7 +899,7 @@ extern "C" int st_plan_set_dist(st_plan* p, const void* uid, int rank, int nrank
     ncclResult_t r = nccl().commInitRank(&comm, nranks, id, rank);
     if (r != ncclSuccess) return fail(ST_ENCCL, "ncclCommInitRank: %s", nccl().errorString(r));
     Dist& D = p->dist;
-    D.mode = Dist::NCCL; D.comm = comm;
+    D.mode = Dist::NCCL; D.nccl_comm = comm;
     D.nz = p->nz; D.P = nranks; D.rank = rank; D.g = g; D.z0 = z0; D.nzl = nzl; D.nzb = nzl + 2 * g;
     D.nranks = nranks;
     p->fl2_of = nullptr; p->flags_checked = nullptr;

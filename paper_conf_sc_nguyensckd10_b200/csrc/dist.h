@@ -30,6 +30,7 @@ struct SlabView {
     const uint8_t* flags = nullptr;   // LBM flags of this slab buffer (nzb planes)
     uint8_t* fl2 = nullptr;           // LBM neighbour-flag buffer of this slab (nzb planes)
     bool single = true;           // the whole grid in one buffer
+    int grid_cap = 0;             // >0: leave SMs free (overlapped NCCL kernels)
     cudaStream_t stream = nullptr;
 };
 
@@ -61,7 +62,7 @@ struct Dist {
     int z0 = 0, nzl = 0, nzb = 0;        // this rank's slab (NCCL) / whole grid (SINGLE)
     int nranks = 1;                       // P for NCCL, 1 otherwise (caller-visible)
 #if ST_HAVE_NCCL
-    ncclComm_t comm = nullptr;
+    ncclComm_t nccl_comm = nullptr;
 #endif
     struct Slab {
         int z0 = 0, nzl = 0, nzb = 0;
@@ -70,6 +71,8 @@ struct Dist {
         uint8_t* fl2 = nullptr;
     };
     std::vector<Slab> slabs;              // LOOPBACK
+    cudaStream_t comm = nullptr;          // ghost-exchange stream (overlapped with interior sweeps)
+    cudaEvent_t ev_b = nullptr, ev_x = nullptr;
     size_t slab_cell_bytes = 0;
     int slab_ncomp = 0;
 
