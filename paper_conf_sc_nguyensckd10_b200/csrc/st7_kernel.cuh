@@ -156,10 +156,11 @@ __device__ __forceinline__ void st7_level(const Blk<float, VY>& ZM, const Blk<fl
         const float right = __shfl_down_sync(0xffffffffu, C.a[j].x, 1, NTX);  // x0 + 4
         const float2 yma = j > 0 ? C.a[j - 1] : top.a, ypa = j < VY - 1 ? C.a[j + 1] : bot.a;
         const float2 ymb = j > 0 ? C.b[j - 1] : top.b, ypb = j < VY - 1 ? C.b[j + 1] : bot.b;
-        // X sums: (x-1 + x+1) for (c0, c1) = (L, c0) + (c1, c2); for (c2, c3) = (c1, c2) + (c3, R)
-        const float2 mid = make_float2(C.a[j].y, C.b[j].x);
-        const float2 sxa = __fadd2_rn(make_float2(left, C.a[j].x), mid);
-        const float2 sxb = __fadd2_rn(mid, make_float2(C.b[j].y, right));
+        // X sums (x-1 + x+1): (c0, c1) -> (c1 + L, c0 + c2) = swap(a) + (L, c2);
+        // (c2, c3) -> (c3 + c1, c2 + R) = swap(b) + (c1, R).  The swapped pairs are
+        // operand swizzles (.LO_HI), so only one half of each constructed pair moves.
+        const float2 sxa = __fadd2_rn(make_float2(C.a[j].y, C.a[j].x), make_float2(left, C.b[j].x));
+        const float2 sxb = __fadd2_rn(make_float2(C.b[j].y, C.b[j].x), make_float2(C.a[j].y, right));
         float2 sa, sb;
         if (EXACT) {   // oracle order (X2)
             sa = __fadd2_rn(__fadd2_rn(sxa, __fadd2_rn(yma, ypa)), __fadd2_rn(ZM.a[j], ZP.a[j]));
