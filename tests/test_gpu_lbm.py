@@ -91,3 +91,16 @@ def test_bad_omega():
     f0 = stgen.lbm_rest(32, 16, 12, np.float32)
     with pytest.raises(st.StError):
         run_gpu(f0, flags, 2.0, 2)
+
+
+@pytest.mark.parametrize("dim_T", [1, 2])
+def test_config2_lbm_256_full_lattice(oracle_lib, dim_T):
+    # configs[2] size: 256^3 lid-driven cavity, random populations, every cell compared
+    n, T = 256, 2
+    flags = stgen.cavity_flags(n, n, n)
+    f0 = stgen.lbm_random(n, n, n, 3, np.float32)
+    ref = oracle_lib.lbm(f0, flags, 1.6, T)
+    got = run_gpu(f0, flags, 1.6, T, dim_T=dim_T)
+    assert relerr(got, ref) <= TOL[np.float32]
+    got = run_gpu(f0, flags, 1.6, T, dim_T=dim_T, exact=True)
+    assert np.array_equal(got, ref)

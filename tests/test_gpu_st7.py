@@ -110,11 +110,25 @@ def test_errors():
             p.st7(x, np.empty((64, 64, 64), np.float32), 0.4, 0.1, 1)  # mixed host/device
 
 
-@pytest.mark.parametrize("dtype", [np.float32, np.float64])
-def test_config2_256_sampled(oracle_lib, dtype):
-    # BASELINE configs[1] size in the launch configuration bench.py times (dim_T=4 f32)
-    n, T = 256, 20
+@pytest.mark.parametrize("dtype,dim_T", [(np.float32, 3), (np.float32, 4), (np.float64, 3)])
+def test_config2_256_full_grid(oracle_lib, dtype, dim_T):
+    # BASELINE configs[1] exactly as bench.py times it: 256^3, T = 100, seed 2
+    n, T = 256, 100
     a = stgen.grid7(n, n, n, 2, dtype)
     ref = oracle_lib.st7(a, 0.4, 0.1, T)
-    got, info = run_gpu(a, 0.4, 0.1, T, 4 if dtype == np.float32 else 2)
-    assert relerr(got, ref) <= TOL[dtype] * 2
+    got, info = run_gpu(a, 0.4, 0.1, T, dim_T)
+    assert relerr(got, ref) <= TOL[dtype]
+    got, _ = run_gpu(a, 0.4, 0.1, T, dim_T, exact=True)
+    assert np.array_equal(got, ref)
+
+
+def test_config3_512_full_grid(oracle_lib):
+    # configs[3] per-GPU size in the launch configuration bench.py's 512^3 extra times (dim_T 4)
+    n, T = 512, 8
+    a = stgen.grid7(n, n, n, 4, np.float32)
+    ref = oracle_lib.st7(a, 0.4, 0.1, T)
+    got, info = run_gpu(a, 0.4, 0.1, T, 4)
+    assert info["dim_t_sweep"] == 4
+    assert relerr(got, ref) <= TOL[np.float32]
+    got, _ = run_gpu(a, 0.4, 0.1, T, 4, exact=True)
+    assert np.array_equal(got, ref)
