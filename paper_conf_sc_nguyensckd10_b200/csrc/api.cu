@@ -81,6 +81,7 @@ static int encode_3d(CUtensorMap* map, const void* base, st_dtype dt, int nx, in
 struct Geo7 {
     int d = 0, VY = 0, NTX = 0, VX = 0, TX = 0, NTY = 0, TY = 0;
     int hx = 0, wx = 0, wy = 0, tiles_x = 0, tiles_y = 0, threads = 0, grid = 0, maxt = 0, ring = 4;
+    bool split = false;   // warp-specialised two-group kernel (st7_split.cuh)
     size_t smem = 0;
     double kappa = 0;
     St7LaunchFn fn = nullptr;
@@ -108,7 +109,6 @@ struct st_plan {
     const void* flags_checked = nullptr;
     uint8_t* fl2 = nullptr;          // flags | 0x80 (FLUID next to non-FLUID), lbm_35d input
     size_t fl2_bytes = 0;
-    const void* fl2_of = nullptr;
     // distribution (Z slabs)
     Dist dist;
     std::map<int, Geo7> geo7;  // by depth
@@ -123,10 +123,13 @@ static int max_lbm_depth(const st_plan* p);
 // the register budget of each (D, VY, MAXT) instantiation, from ptxas -v
 // (no spills): 512 threads cap registers at 128 and double the resident
 // warps; 256 threads allow 255 registers for the deeper Z windows.
-static void variant_for(st_dtype dt, int d, int& vy, int& maxt) {
-    if (const char* e = getenv("ST_VARIANT")) {  // "VYxMAXT", e.g. 4x256 (tuning only)
+static void variant_for(st_dtype dt, int d, int& vy, int& maxt, bool& split) {
+    split = false;
+    if (const char* e = getenv("ST_VARIANT")) {  // "VYxMAXT[s]", e.g. 4x256, 4x512s (tuning only)
         int a = 0, b = 0;
-        if (sscanf(e, "%dx%d", &a, &b) == 2) { vy = a; maxt = b; return; }
+        char c = 0;
+        const int n = sscanf(e, "%dx%d%c", &a, &b, &c);
+        if (n >= 2) { vy = a; maxt = b; split = n == 3 && c == 's' && d >= 2 && d <= 6; return; }
     }
     // measured on B200 (tools/quickbench.py): VY=4 / 256 threads is fastest
     // while it fits without spills; deeper sweeps need the smaller block
@@ -134,12 +137,19 @@ static void variant_for(st_dtype dt, int d, int& vy, int& maxt) {
     vy = d <= 3 ? 4 : 2; maxt = 256;
 }
 
-static St7LaunchFn lookup7(st_dtype dt, bool exact, int d, int vy, int maxt) {
+static St7LaunchFn lookup7(st_dtype dt, bool exact, int d, int vy, int maxt, bool split) {
+    if (split) {
+        if (dt == ST_F32) return exact ? st7s_lookup_f32_exact(d, vy, maxt) : st7s_lookup_f32_fast(d, vy, maxt);
+        return exact ? st7s_lookup_f64_exact(d, vy, maxt) : st7s_lookup_f64_fast(d, vy, maxt);
+    }
     if (dt == ST_F32) return exact ? st7_lookup_f32_exact(d, vy, maxt) : st7_lookup_f32_fast(d, vy, maxt);
     return exact ? st7_lookup_f64_exact(d, vy, maxt) : st7_lookup_f64_fast(d, vy, maxt);
 }
 
 static size_t smem7(const Geo7& g, st_dtype dt, int ring) {
+    if (g.split)   // TMA ring + 4-plane hand-off ring + exchange [D-2][2][2][MAXT/2] + mbarriers
+        return (size_t)(ring + 4) * g.TX * g.TY * esize(dt) + (size_t)(g.d > 2 ? g.d - 2 : 0) * 4 * (g.maxt / 2) * 16 +
+               ring * 8;
     // TMA ring + row exchange [D-1][2][2][MAXT] x 16 B + mbarriers
     return (size_t)ring * g.TX * g.TY * esize(dt) + (size_t)(g.d > 1 ? g.d - 1 : 0) * 4 * g.maxt * 16 +
            ring * 8;
@@ -155,18 +165,19 @@ static int plan7(st_plan* p, int d, int nzo, Geo7& g) {
     g.VX = p->dtype == ST_F32 ? 4 : 2;
     g.NTX = p->dtype == ST_F32 ? 16 : 32;
     g.TX = g.NTX * g.VX;
-    variant_for(p->dtype, d, g.VY, g.maxt);
+    variant_for(p->dtype, d, g.VY, g.maxt, g.split);
     g.hx = (d + g.VX - 1) / g.VX * g.VX;
     g.wx = (g.TX - g.hx - d) & ~(g.VX - 1);
     if (g.wx < g.VX) return fail(ST_EUNSUPPORTED, "dim_T %d too deep for a %d-wide tile", d, g.TX);
     g.tiles_x = (p->nx + g.wx - 1) / g.wx;
-    const int ntymax = g.maxt / g.NTX;
+    const int ntymax = g.maxt / (g.split ? 2 : 1) / g.NTX;   // thread rows per (group of the) CTA
     long best = -1;
     for (int nty = 2; nty <= ntymax; ++nty) {
+        if (g.split && (g.NTX * nty) % 32) continue;   // groups must be whole warps
         Geo7 c = g;
         c.NTY = nty;
         c.TY = nty * c.VY;
-        c.threads = c.NTX * nty;
+        c.threads = c.NTX * nty * (c.split ? 2 : 1);
         c.wy = c.TY - 2 * d;
         if (c.wy < 1) continue;
         c.tiles_y = (p->ny + c.wy - 1) / c.wy;
@@ -188,14 +199,14 @@ static int plan7(st_plan* p, int d, int nzo, Geo7& g) {
     const long long work = (long long)g.tiles_x * g.tiles_y * nzo;
     g.grid = (int)std::min<long long>(p->sms, std::max<long long>(work, 1));
     g.kappa = (double)g.tiles_x * g.TX * g.tiles_y * g.TY / ((double)p->nx * p->ny);
-    g.fn = lookup7(p->dtype, p->exact, d, g.VY, g.maxt);
+    g.fn = lookup7(p->dtype, p->exact, d, g.VY, g.maxt, g.split);
     if (!g.fn) return fail(ST_EUNSUPPORTED, "no kernel for dim_T %d", d);
     return ST_OK;
 }
 
 static int get_geo7(st_plan* p, int d, int nzo, Geo7*& out) {
     auto it = p->geo7.find(d);
-    if (it == p->geo7.end() || it->second.fn != lookup7(p->dtype, p->exact, d, it->second.VY, it->second.maxt)) {
+    if (it == p->geo7.end() || it->second.fn != lookup7(p->dtype, p->exact, d, it->second.VY, it->second.maxt, it->second.split)) {
         Geo7 g;
         int rc = plan7(p, d, nzo, g);
         if (rc) return rc;
@@ -318,7 +329,7 @@ extern "C" int st_plan_get_info(const st_plan* p, int lbm, st_plan_info* info) {
     const Geo7& g = it->second;
     info->tile_x = g.TX; info->tile_y = g.TY; info->out_x = g.wx; info->out_y = g.wy;
     info->tiles_x = g.tiles_x; info->tiles_y = g.tiles_y; info->ctas = g.grid; info->threads = g.threads;
-    info->smem_bytes = (int)g.smem; info->kappa = g.kappa; info->kernel = g.VY * 1000 + g.maxt;
+    info->smem_bytes = (int)g.smem; info->kappa = g.kappa; info->kernel = g.VY * 1000 + g.maxt + (g.split ? 100000 : 0);
     info->dim_t_sweep = p->dimK;
     info->ring = g.ring;
     return ST_OK;
@@ -759,7 +770,8 @@ static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T
     // dim_T = 1: the fused push kernel (fastest measured on B200); dim_T >= 2:
     // the on-chip multi-level sweep lbm_35d (ST_LBM_35D=1 forces it for dim_T = 1)
     const bool push = max_lbm_depth(p) == 1 && getenv("ST_LBM_35D") == nullptr && p->dist.mode == Dist::SINGLE;
-    if (!push && p->dist.mode != Dist::LOOPBACK && p->fl2_of != flags) {   // neighbour-flag prepass (once per flags pointer)
+    // neighbour-flag prepass, every call (a reused flags pointer may hold new contents; ~1 pass over the flags)
+    if (!push && p->dist.mode != Dist::LOOPBACK) {
         const size_t cells = (size_t)p->nx * p->ny * p->dist.nzb;
         if (p->fl2_bytes < cells) {
             if (p->fl2) cudaFree(p->fl2);
@@ -769,7 +781,6 @@ static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T
         }
         cudaError_t e = lbm_fl2(flags, p->fl2, p->nx, p->ny, p->dist.nzb, p->stream);
         if (e != cudaSuccess) return fail(ST_ECUDA, "fl2 prepass: %s", cudaGetErrorString(e));
-        p->fl2_of = flags;
     }
     std::vector<int> ds = push ? std::vector<int>(T, 1) : sweep_depths(T, max_lbm_depth(p));
     rc = run_sweeps(p, ds, fsrc, fdst, 19, flags, [&](const void* a, void* b, int d, const SlabView& sv) {
@@ -807,7 +818,6 @@ extern "C" int lbm_d3q19_run(st_plan* p, void* fsrc, void* fdst, double omega, i
     CUDA_TRY(cudaMemcpyAsync(p->hbuf[0], fsrc, n, cudaMemcpyHostToDevice, p->stream));
     CUDA_TRY(cudaMemcpyAsync(p->hflags, flags, cells, cudaMemcpyHostToDevice, p->stream));
     p->flags_checked = nullptr;  // staging buffer content changes per call
-    p->fl2_of = nullptr;
     rc = runlbm_device(p, p->hbuf[0], p->hbuf[1], omega, T, p->hflags);
     if (rc) return rc;
     CUDA_TRY(cudaMemcpyAsync(fdst, p->hbuf[1], n, cudaMemcpyDeviceToHost, p->stream));
@@ -902,7 +912,7 @@ extern "C" int st_plan_set_dist(st_plan* p, const void* uid, int rank, int nrank
     D.mode = Dist::NCCL; D.nccl_comm = comm;
     D.nz = p->nz; D.P = nranks; D.rank = rank; D.g = g; D.z0 = z0; D.nzl = nzl; D.nzb = nzl + 2 * g;
     D.nranks = nranks;
-    p->fl2_of = nullptr; p->flags_checked = nullptr;
+    p->flags_checked = nullptr;
     return ST_OK;
 #else
     (void)uid;

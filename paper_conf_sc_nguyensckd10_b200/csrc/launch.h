@@ -16,6 +16,11 @@ St7LaunchFn st7_lookup_f32_fast(int D, int VY, int MAXT);
 St7LaunchFn st7_lookup_f32_exact(int D, int VY, int MAXT);
 St7LaunchFn st7_lookup_f64_fast(int D, int VY, int MAXT);
 St7LaunchFn st7_lookup_f64_exact(int D, int VY, int MAXT);
+// warp-specialised two-group variant (st7_split.cuh), D in [2, 6]
+St7LaunchFn st7s_lookup_f32_fast(int D, int VY, int MAXT);
+St7LaunchFn st7s_lookup_f32_exact(int D, int VY, int MAXT);
+St7LaunchFn st7s_lookup_f64_fast(int D, int VY, int MAXT);
+St7LaunchFn st7s_lookup_f64_exact(int D, int VY, int MAXT);
 
 cudaError_t lbm_push_launch(int dtype, bool exact, const void* src, void* dst, const uint8_t* flags,
                             const LbmParams& p, int grid, cudaStream_t s);

@@ -46,25 +46,27 @@ cudaError_t lbm35_launch(int dtype, bool exact, int D, const Lbm35Params& p, int
 
 // fl2 = flags | 0x80 where a FLUID cell has a non-FLUID (or out-of-lattice) neighbour
 __global__ void lbm_fl2_kernel(const uint8_t* __restrict__ flags, uint8_t* __restrict__ fl2, int nx, int ny, int nz) {
-    const size_t plane = (size_t)nx * ny, n = plane * nz;
-    for (size_t c = blockIdx.x * (size_t)blockDim.x + threadIdx.x; c < n; c += (size_t)gridDim.x * blockDim.x) {
-        const int x = (int)(c % nx), y = (int)((c / nx) % ny), z = (int)(c / plane);
-        uint8_t f = flags[c];
-        if (f == 0) {
-            bool nb = false;
-            for (int i = 1; i < 19; ++i) {
-                const int X = x + c_ex[i], Y = y + c_ey[i], Z = z + c_ez[i];
-                if (X < 0 || Y < 0 || Z < 0 || X >= nx || Y >= ny || Z >= nz) { nb = true; break; }
-                if (flags[(size_t)Z * plane + (size_t)Y * nx + X] != 0) { nb = true; break; }
-            }
-            if (nb) f |= 0x80;
+    // grid (ceil(nx / 256), ny, nz): no index divisions
+    const int x = blockIdx.x * blockDim.x + threadIdx.x, y = blockIdx.y, z = blockIdx.z;
+    if (x >= nx) return;
+    const size_t plane = (size_t)nx * ny;
+    const size_t c = (size_t)z * plane + (size_t)y * nx + x;
+    uint8_t f = flags[c];
+    if (f == 0) {
+        bool nb = x == 0 || y == 0 || z == 0 || x == nx - 1 || y == ny - 1 || z == nz - 1;
+#pragma unroll
+        for (int i = 1; i < 19; ++i) {
+            if (nb) break;
+            nb = flags[(size_t)((long long)c + c_ex[i] + (long long)c_ey[i] * nx + (long long)c_ez[i] * (long long)plane)] != 0;
         }
-        fl2[c] = f;
+        if (nb) f |= 0x80;
     }
+    fl2[c] = f;
 }
 
 cudaError_t lbm_fl2(const uint8_t* flags, uint8_t* fl2, int nx, int ny, int nz, cudaStream_t s) {
-    lbm_fl2_kernel<<<148 * 8, 256, 0, s>>>(flags, fl2, nx, ny, nz);
+    if (nz > 65535 || ny > 65535) return cudaErrorInvalidValue;
+    lbm_fl2_kernel<<<dim3((nx + 255) / 256, ny, nz), 256, 0, s>>>(flags, fl2, nx, ny, nz);
     return cudaGetLastError();
 }
 

@@ -1,6 +1,7 @@
 // st7_inst.cu — instantiates st7_35d_kernel for one (dtype, mode); compiled
 // once per combination with -DST_T=float|double -DST_EXACT=0|1.
 #include "launch.h"
+#include "st7_split.cuh"
 
 #ifndef ST_T
 #define ST_T float
@@ -52,6 +53,28 @@ St7LaunchFn pick(int D) {
     }
 }
 
+template <int D, int VY, int MAXT>
+cudaError_t launch_split(const CUtensorMap* map, const St7Params& p, int grid, int threads, size_t smem,
+                         cudaStream_t s) {
+    auto k = st7_35d_split_kernel<TT, D, (D + 1) / 2, NTX, VY, ST_EXACT != 0, MAXT>;
+    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    k<<<grid, threads, smem, s>>>(*map, p);
+    return cudaGetLastError();
+}
+
+template <int VY, int MAXT>
+St7LaunchFn pick_split(int D) {
+    switch (D) {
+        case 2: return launch_split<2, VY, MAXT>;
+        case 3: return launch_split<3, VY, MAXT>;
+        case 4: return launch_split<4, VY, MAXT>;
+        case 5: return launch_split<5, VY, MAXT>;
+        case 6: return launch_split<6, VY, MAXT>;
+        default: return nullptr;
+    }
+}
+
 }  // namespace ST_UNIT_NS
 using namespace ST_UNIT_NS;
 
@@ -66,4 +89,13 @@ St7LaunchFn ST_FN(int D, int VY, int MAXT) {
     return nullptr;
 }
 
+}  // namespace st35d
+
+namespace st35d {
+#define ST_SFN ST_CAT(ST_CAT(ST_CAT(st7s_lookup_, ST_TNAME), _), ST_MODE)
+St7LaunchFn ST_SFN(int D, int VY, int MAXT) {
+    if (VY == 2 && MAXT == 512) return pick_split<2, 512>(D);
+    if (VY == 4 && MAXT == 384) return pick_split<4, 384>(D);
+    return nullptr;
+}
 }  // namespace st35d

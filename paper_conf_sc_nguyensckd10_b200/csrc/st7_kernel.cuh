@@ -135,12 +135,19 @@ template <> struct Coef<float> {
         k.beB = make_float2(xfix & 4 ? 0.f : be, xfix & 8 ? 0.f : be);
         return k;
     }
+    // field-wise select (a ?: on the structs would take their addresses -> local memory)
+    static __device__ __forceinline__ Coef sel(bool f, const Coef& x, const Coef& y) {
+        return Coef{f ? x.alA : y.alA, f ? x.beA : y.beA, f ? x.alB : y.alB, f ? x.beB : y.beB};
+    }
 };
 template <> struct Coef<double> {
     double al[2], be[2];
     static __device__ __forceinline__ Coef fixed() { return Coef{{1.0, 1.0}, {0.0, 0.0}}; }
     static __device__ __forceinline__ Coef make(double al, double be, uint32_t xfix) {
         return Coef{{xfix & 1 ? 1.0 : al, xfix & 2 ? 1.0 : al}, {xfix & 1 ? 0.0 : be, xfix & 2 ? 0.0 : be}};
+    }
+    static __device__ __forceinline__ Coef sel(bool f, const Coef& x, const Coef& y) {
+        return Coef{{f ? x.al[0] : y.al[0], f ? x.al[1] : y.al[1]}, {f ? x.be[0] : y.be[0], f ? x.be[1] : y.be[1]}};
     }
 };
 
