@@ -15,7 +15,7 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libst35d.so")
+LIB_PATH = os.environ.get("ST35D_LIB") or os.path.join(_HERE, "libst35d.so")   # override: A/B tuning builds
 
 ST_F32, ST_F64 = 0, 1
 ST_OK, ST_EINVAL, ST_ENOMEM, ST_ECUDA, ST_ENCCL, ST_EUNSUPPORTED = 0, -1, -2, -3, -4, -5

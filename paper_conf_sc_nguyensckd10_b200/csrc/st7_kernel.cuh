@@ -151,16 +151,41 @@ template <> struct Coef<double> {
     }
 };
 
+// X neighbours of a block's rows from the neighbouring lanes (x0 - 1 and x0 + VX):
+// issued one level ahead by the kernel so the shuffle latency overlaps a level
+template <typename T, int VY> struct XN { T l[VY], r[VY]; };
+template <int NTX, int VY>
+__device__ __forceinline__ XN<float, VY> xshuf(const Blk<float, VY>& C) {
+    XN<float, VY> x;
+#pragma unroll
+    for (int j = 0; j < VY; ++j) {
+        x.l[j] = __shfl_up_sync(0xffffffffu, C.b[j].y, 1, NTX);
+        x.r[j] = __shfl_down_sync(0xffffffffu, C.a[j].x, 1, NTX);
+    }
+    return x;
+}
+template <int NTX, int VY>
+__device__ __forceinline__ XN<double, VY> xshuf(const Blk<double, VY>& C) {
+    XN<double, VY> x;
+#pragma unroll
+    for (int j = 0; j < VY; ++j) {
+        x.l[j] = __shfl_up_sync(0xffffffffu, C.v[j][1], 1, NTX);
+        x.r[j] = __shfl_down_sync(0xffffffffu, C.v[j][0], 1, NTX);
+    }
+    return x;
+}
+
 // one level of the sweep for one thread's block: R = stencil(ZM, C, ZP)
-template <int NTX, int VY, bool EXACT>
+// (PRE: X neighbours pre-shuffled in xn; otherwise shuffled here, row by row)
+template <int NTX, int VY, bool EXACT, bool PRE = true>
 __device__ __forceinline__ void st7_level(const Blk<float, VY>& ZM, const Blk<float, VY>& C,
-                                          const Blk<float, VY>& ZP, const Row<float>& top,
+                                          const Blk<float, VY>& ZP, const XN<float, VY>& xn, const Row<float>& top,
                                           const Row<float>& bot, const Coef<float>& k, bool yslow,
                                           uint32_t rowfix, Blk<float, VY>& R) {
 #pragma unroll
     for (int j = 0; j < VY; ++j) {
-        const float left = __shfl_up_sync(0xffffffffu, C.b[j].y, 1, NTX);     // x0 - 1
-        const float right = __shfl_down_sync(0xffffffffu, C.a[j].x, 1, NTX);  // x0 + 4
+        const float left = PRE ? xn.l[j] : __shfl_up_sync(0xffffffffu, C.b[j].y, 1, NTX);     // x0 - 1
+        const float right = PRE ? xn.r[j] : __shfl_down_sync(0xffffffffu, C.a[j].x, 1, NTX);  // x0 + 4
         const float2 yma = j > 0 ? C.a[j - 1] : top.a, ypa = j < VY - 1 ? C.a[j + 1] : bot.a;
         const float2 ymb = j > 0 ? C.b[j - 1] : top.b, ypb = j < VY - 1 ? C.b[j + 1] : bot.b;
         // X sums (x-1 + x+1): (c0, c1) -> (c1 + L, c0 + c2) = swap(a) + (L, c2);
@@ -193,15 +218,15 @@ __device__ __forceinline__ void st7_level(const Blk<float, VY>& ZM, const Blk<fl
     }
 }
 
-template <int NTX, int VY, bool EXACT>
+template <int NTX, int VY, bool EXACT, bool PRE = true>
 __device__ __forceinline__ void st7_level(const Blk<double, VY>& ZM, const Blk<double, VY>& C,
-                                          const Blk<double, VY>& ZP, const Row<double>& top,
+                                          const Blk<double, VY>& ZP, const XN<double, VY>& xn, const Row<double>& top,
                                           const Row<double>& bot, const Coef<double>& k, bool yslow,
                                           uint32_t rowfix, Blk<double, VY>& R) {
 #pragma unroll
     for (int j = 0; j < VY; ++j) {
-        const double left = __shfl_up_sync(0xffffffffu, C.v[j][1], 1, NTX);
-        const double right = __shfl_down_sync(0xffffffffu, C.v[j][0], 1, NTX);
+        const double left = PRE ? xn.l[j] : __shfl_up_sync(0xffffffffu, C.v[j][1], 1, NTX);
+        const double right = PRE ? xn.r[j] : __shfl_down_sync(0xffffffffu, C.v[j][0], 1, NTX);
 #pragma unroll
         for (int i = 0; i < 2; ++i) {
             const double c = C.v[j][i];
@@ -218,6 +243,13 @@ __device__ __forceinline__ void st7_level(const Blk<double, VY>& ZM, const Blk<d
         for (int j = 0; j < VY; ++j)
             if (rowfix & (1u << j)) { R.v[j][0] = C.v[j][0]; R.v[j][1] = C.v[j][1]; }
     }
+}
+
+template <int NTX, int VY, bool EXACT, typename T>
+__device__ __forceinline__ void st7_level(const Blk<T, VY>& ZM, const Blk<T, VY>& C, const Blk<T, VY>& ZP,
+                                          const Row<T>& top, const Row<T>& bot, const Coef<T>& k, bool yslow,
+                                          uint32_t rowfix, Blk<T, VY>& R) {
+    st7_level<NTX, VY, EXACT, false>(ZM, C, ZP, XN<T, VY>{}, top, bot, k, yslow, rowfix, R);
 }
 
 template <typename T, int D, int NTX, int VY, bool EXACT, int MAXT>
@@ -351,62 +383,130 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
             // level 0: plane r has landed in the ring
             if (STEADY || r <= rl1) mbar_wait(&bars[slot_r], par_r);
             const int rpar = r & 1;
-            // levels 1..D: level l computes plane z = r - l
-#pragma unroll
-            for (int l = 1; l <= D; ++l) {
-                if (p.dbg & 1) break;   // tuning only: stream the planes without computing
-                const int z = r - l;
-                bool zfix = false;
-                if (!STEADY) {
-                    const int lo = max(za - (D - l), zmin), hi = min(zb - 1 + (D - l), zmax);
-                    if (z < lo || z > hi) continue;
-                    const int zg = p.zbase + z;
-                    zfix = (zg == 0) || (zg == p.nzg - 1);
-                }
-                const int zpar = rpar ^ (l & 1);
-                Row<T> top, bot;
-                if (l == 1) {   // level-0 neighbours of plane r-1 straight from the TMA ring
-                    const T* sl = ring + slot_m1 * slot_elems;
-                    top = row_nat(sl + top_off);
-                    bot = row_nat(sl + bot_off);
-                } else {        // rows exchanged by the blocks above / below in round r-1
-                    const int o = ((l - 2) * 4 + zpar * 2) * MAXT;
-                    top = row_x(xtop + o);
-                    bot = row_x(xbot + o);
-                }
-                B& dst = l < D ? pl[l < D ? l : 1][NEW] : outv;
-                if (l == 1) {   // level-0 planes r-2, r-1, r of my block straight from the ring
-                    B zm, c, zp;
-                    const T* s2 = ring + slot_m2 * slot_elems + my_off;
-                    const T* s1 = ring + slot_m1 * slot_elems + my_off;
-                    const T* s0 = ring + slot_r * slot_elems + my_off;
-#pragma unroll
-                    for (int j = 0; j < VY; ++j) {
-                        zm.load_nat(j, s2 + j * TX);
-                        c.load_nat(j, s1 + j * TX);
-                        zp.load_nat(j, s0 + j * TX);
+            // (The look-ahead exchange is measured faster for FP64 and VY = 2; the
+            // FP32 VY = 4 blocks have no registers to spare and exchange per level.)
+            if constexpr (sizeof(T) == 8 || VY == 2) {
+                // levels 1..D: level l computes plane z = r - l.  The X-neighbour
+                // shuffles and exchange-row loads of level l+1 (whose centre plane
+                // pl[l][CUR] exists since round r-1) are issued before level l computes.
+                XN<T, VY> xnn;
+                Row<T> tnn, bnn;
+    #pragma unroll
+                for (int l = 1; l <= D; ++l) {
+                    if (p.dbg & 1) break;   // tuning only: stream the planes without computing
+                    const int z = r - l;
+                    const int zpar = rpar ^ (l & 1);
+                    const XN<T, VY> xnl = xnn;
+                    const Row<T> tl = tnn, bl = bnn;
+                    if (l < D) {
+                        xnn = xshuf<NTX, VY>(pl[l][CUR]);
+                        const int o = ((l - 1) * 4 + (zpar ^ 1) * 2) * MAXT;
+                        tnn = row_x(xtop + o);
+                        bnn = row_x(xbot + o);
                     }
-                    if (!STEADY && zfix)
-                        st7_level<NTX, VY, EXACT>(zm, c, zp, top, bot, Coef<T>::fixed(), yslow, rowfix, dst);
-                    else
-                        st7_level<NTX, VY, EXACT>(zm, c, zp, top, bot, kc, yslow, rowfix, dst);
-                } else {
-                    const int lp = l > 1 ? l - 1 : 1;
-                    if (!STEADY && zfix)
-                        st7_level<NTX, VY, EXACT>(pl[lp][PREV], pl[lp][CUR], pl[lp][NEW], top, bot,
-                                                  Coef<T>::fixed(), yslow, rowfix, dst);
-                    else
-                        st7_level<NTX, VY, EXACT>(pl[lp][PREV], pl[lp][CUR], pl[lp][NEW], top, bot, kc,
-                                                  yslow, rowfix, dst);
+                    bool zfix = false;
+                    if (!STEADY) {
+                        const int lo = max(za - (D - l), zmin), hi = min(zb - 1 + (D - l), zmax);
+                        if (z < lo || z > hi) continue;
+                        const int zg = p.zbase + z;
+                        zfix = (zg == 0) || (zg == p.nzg - 1);
+                    }
+                    B& dst = l < D ? pl[l < D ? l : 1][NEW] : outv;
+                    if (l == 1) {   // level-0 planes r-2, r-1, r of my block straight from the TMA ring
+                        const T* sl = ring + slot_m1 * slot_elems;   // level-0 neighbour rows of plane r-1
+                        const Row<T> top = row_nat(sl + top_off), bot = row_nat(sl + bot_off);
+                        B zm, c, zp;
+                        const T* s2 = ring + slot_m2 * slot_elems + my_off;
+                        const T* s1 = ring + slot_m1 * slot_elems + my_off;
+                        const T* s0 = ring + slot_r * slot_elems + my_off;
+    #pragma unroll
+                        for (int j = 0; j < VY; ++j) {
+                            zm.load_nat(j, s2 + j * TX);
+                            c.load_nat(j, s1 + j * TX);
+                            zp.load_nat(j, s0 + j * TX);
+                        }
+                        const XN<T, VY> xc = xshuf<NTX, VY>(c);
+                        if (!STEADY && zfix)
+                            st7_level<NTX, VY, EXACT>(zm, c, zp, xc, top, bot, Coef<T>::fixed(), yslow, rowfix, dst);
+                        else
+                            st7_level<NTX, VY, EXACT>(zm, c, zp, xc, top, bot, kc, yslow, rowfix, dst);
+                    } else {
+                        const int lp = l > 1 ? l - 1 : 1;
+                        if (!STEADY && zfix)
+                            st7_level<NTX, VY, EXACT>(pl[lp][PREV], pl[lp][CUR], pl[lp][NEW], xnl, tl, bl,
+                                                      Coef<T>::fixed(), yslow, rowfix, dst);
+                        else
+                            st7_level<NTX, VY, EXACT>(pl[lp][PREV], pl[lp][CUR], pl[lp][NEW], xnl, tl, bl, kc,
+                                                      yslow, rowfix, dst);
+                    }
+                    if (l < D) {
+                        V* xb = xw + ((l - 1) * 4 + zpar * 2) * MAXT;
+                        dst.store_x(0, xb);
+                        dst.store_x(VY - 1, xb + MAXT);
+                    } else {
+    #pragma unroll
+                        for (int j = 0; j < VY; ++j)
+                            if (rowmask & (1u << j)) outv.store_global(j, pout + j * nxs);
+                    }
                 }
-                if (l < D) {
-                    V* xb = xw + ((l - 1) * 4 + zpar * 2) * MAXT;
-                    dst.store_x(0, xb);
-                    dst.store_x(VY - 1, xb + MAXT);
-                } else {
-#pragma unroll
-                    for (int j = 0; j < VY; ++j)
-                        if (rowmask & (1u << j)) outv.store_global(j, pout + j * nxs);
+            } else {
+                // levels 1..D: level l computes plane z = r - l
+    #pragma unroll
+                for (int l = 1; l <= D; ++l) {
+                    if (p.dbg & 1) break;   // tuning only: stream the planes without computing
+                    const int z = r - l;
+                    bool zfix = false;
+                    if (!STEADY) {
+                        const int lo = max(za - (D - l), zmin), hi = min(zb - 1 + (D - l), zmax);
+                        if (z < lo || z > hi) continue;
+                        const int zg = p.zbase + z;
+                        zfix = (zg == 0) || (zg == p.nzg - 1);
+                    }
+                    const int zpar = rpar ^ (l & 1);
+                    Row<T> top, bot;
+                    if (l == 1) {   // level-0 neighbours of plane r-1 straight from the TMA ring
+                        const T* sl = ring + slot_m1 * slot_elems;
+                        top = row_nat(sl + top_off);
+                        bot = row_nat(sl + bot_off);
+                    } else {        // rows exchanged by the blocks above / below in round r-1
+                        const int o = ((l - 2) * 4 + zpar * 2) * MAXT;
+                        top = row_x(xtop + o);
+                        bot = row_x(xbot + o);
+                    }
+                    B& dst = l < D ? pl[l < D ? l : 1][NEW] : outv;
+                    if (l == 1) {   // level-0 planes r-2, r-1, r of my block straight from the ring
+                        B zm, c, zp;
+                        const T* s2 = ring + slot_m2 * slot_elems + my_off;
+                        const T* s1 = ring + slot_m1 * slot_elems + my_off;
+                        const T* s0 = ring + slot_r * slot_elems + my_off;
+    #pragma unroll
+                        for (int j = 0; j < VY; ++j) {
+                            zm.load_nat(j, s2 + j * TX);
+                            c.load_nat(j, s1 + j * TX);
+                            zp.load_nat(j, s0 + j * TX);
+                        }
+                        if (!STEADY && zfix)
+                            st7_level<NTX, VY, EXACT>(zm, c, zp, top, bot, Coef<T>::fixed(), yslow, rowfix, dst);
+                        else
+                            st7_level<NTX, VY, EXACT>(zm, c, zp, top, bot, kc, yslow, rowfix, dst);
+                    } else {
+                        const int lp = l > 1 ? l - 1 : 1;
+                        if (!STEADY && zfix)
+                            st7_level<NTX, VY, EXACT>(pl[lp][PREV], pl[lp][CUR], pl[lp][NEW], top, bot,
+                                                      Coef<T>::fixed(), yslow, rowfix, dst);
+                        else
+                            st7_level<NTX, VY, EXACT>(pl[lp][PREV], pl[lp][CUR], pl[lp][NEW], top, bot, kc,
+                                                      yslow, rowfix, dst);
+                    }
+                    if (l < D) {
+                        V* xb = xw + ((l - 1) * 4 + zpar * 2) * MAXT;
+                        dst.store_x(0, xb);
+                        dst.store_x(VY - 1, xb + MAXT);
+                    } else {
+    #pragma unroll
+                        for (int j = 0; j < VY; ++j)
+                            if (rowmask & (1u << j)) outv.store_global(j, pout + j * nxs);
+                    }
                 }
             }
             __syncthreads();
