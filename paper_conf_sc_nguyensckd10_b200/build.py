@@ -14,8 +14,13 @@ import sys
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
-BUILD = os.path.join(ROOT, "build", "obj")
-LIB = os.path.join(PKG, "libst35d.so")
+# A/B tuning builds: ST_AB=name builds build/ab/<name>/libst35d.so with the
+# extra -D flags in ST_AB_DEFS (load it with ST35D_LIB=...); the default build
+# is the in-tree product library.
+_AB = os.environ.get("ST_AB")
+BUILD = os.path.join(ROOT, "build", "ab", _AB, "obj") if _AB else os.path.join(ROOT, "build", "obj")
+LIB = os.path.join(ROOT, "build", "ab", _AB, "libst35d.so") if _AB else os.path.join(PKG, "libst35d.so")
+_AB_DEFS = os.environ.get("ST_AB_DEFS", "").split() if _AB else []
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
@@ -37,7 +42,7 @@ def _nccl_include():
 _NCCL_INC = _nccl_include()
 COMMON = ARCH + ["-O3", "-lineinfo", "-std=c++20", "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC",
                  "-Xcompiler", "-ffp-contract=off", "-I", os.path.join(ROOT, "include")] + \
-    (["-DST_HAVE_NCCL=1", "-I", _NCCL_INC] if _NCCL_INC else ["-DST_HAVE_NCCL=0"])
+    (["-DST_HAVE_NCCL=1", "-I", _NCCL_INC] if _NCCL_INC else ["-DST_HAVE_NCCL=0"]) + _AB_DEFS
 
 UNITS = [
     ("api.cu", "api.o", []),
@@ -78,8 +83,13 @@ def build(force: bool = False, verbose: bool = False, jobs: int | None = None) -
     os.makedirs(BUILD, exist_ok=True)
     todo = []
     objs = []
+    only = os.environ.get("ST_AB_ONLY", "").split(",") if _AB else [""]
     for src, obj, extra in UNITS:
         o = os.path.join(BUILD, obj)
+        if _AB and only != [""] and obj[:-2] not in only:   # reuse the product build's object
+            o = os.path.join(ROOT, "build", "obj", obj)
+            objs.append(o)
+            continue
         objs.append(o)
         if force or _stale(o, src):
             todo.append((src, o, extra))

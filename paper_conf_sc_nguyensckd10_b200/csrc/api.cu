@@ -374,6 +374,43 @@ static bool overlap(const void* a, const void* b, size_t n) {
 // ----------------------------------------------------------------------------
 // 7-point
 // ----------------------------------------------------------------------------
+// Flexible load balance over persistent CTAs: the (tile, plane)
+// work items, in tile-major order, are cut into G contiguous ranges of equal
+// COST, where a range pays its planes plus a fixed overhead per tile segment it
+// touches (the 2*dim_T prolog/epilog rounds that fill and drain the on-chip
+// levels, at about half a steady round each, plus the first plane's load
+// latency).  Minimises the largest cost by bisection over a greedy cut.
+static void split_work(int ntiles, int nzo, int d, int G, int* split) {
+    const long long work = (long long)ntiles * nzo;
+    const long long ovh = d + 2;
+    auto cuts = [&](long long C, int* out) {   // CTAs needed with per-CTA cost cap C
+        if (C <= ovh) return G + 1;             // no CTA could take a plane
+        long long it = 0;
+        int b = 0;
+        while (it < work) {
+            if (out) out[b] = (int)it;
+            ++b;
+            long long budget = C;
+            while (it < work) {
+                const long long in_tile = (it / nzo + 1) * nzo - it;
+                if (budget <= ovh) break;
+                const long long take = std::min(in_tile, budget - ovh);
+                it += take;
+                budget -= take + ovh;
+                if (take < in_tile) break;
+            }
+        }
+        return b;
+    };
+    long long lo = 1, hi = work + ovh * (ntiles + 1);
+    while (lo < hi) {
+        const long long mid = (lo + hi) / 2;
+        if (cuts(mid, nullptr) <= G) hi = mid; else lo = mid + 1;
+    }
+    const int used = cuts(lo, split);
+    for (int b = used; b <= G; ++b) split[b] = (int)work;   // idle CTAs (tiny grids) get empty ranges
+}
+
 static int launch7(st_plan* p, const void* src, void* dst, int d, double alpha, double beta, const SlabView& sv) {
     Geo7* g = nullptr;
     int rc = get_geo7(p, d, sv.zb - sv.za, g);
@@ -392,7 +429,8 @@ static int launch7(st_plan* p, const void* src, void* dst, int d, double alpha, 
     if (const char* e = getenv("ST_DBG")) prm.dbg = atoi(e);
     prm.alpha = alpha; prm.beta = beta;
     if (prm.work <= 0) return ST_OK;
-    const int grid = sv.grid_cap > 0 ? std::min(g->grid, sv.grid_cap) : g->grid;
+    const int grid = std::min(sv.grid_cap > 0 ? std::min(g->grid, sv.grid_cap) : g->grid, ST7_MAX_GRID);
+    split_work(prm.ntiles, sv.zb - sv.za, d, grid, prm.split);
     cudaError_t e = g->fn(&map, prm, grid, g->threads, g->smem, sv.stream ? sv.stream : p->stream);
     if (e != cudaSuccess) return fail(ST_ECUDA, "st7 launch (d=%d): %s", d, cudaGetErrorString(e));
     ++p->launches;

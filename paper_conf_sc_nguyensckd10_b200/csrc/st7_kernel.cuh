@@ -28,7 +28,16 @@
 #include <type_traits>
 #include "common.cuh"
 
+#ifndef ST_ZLAST
+#define ST_ZLAST 0
+#endif
+#ifndef ST7_DBG
+#define ST7_DBG 0
+#endif
+
 namespace st35d {
+
+constexpr int ST7_MAX_GRID = 160;   // >= SM count (148 on B200); one persistent CTA per SM
 
 struct St7Params {
     void* out;
@@ -44,6 +53,7 @@ struct St7Params {
     int ring;          // TMA ring slots (<= ST7_RING_MAX); ring - 2 planes are prefetched ahead
     int dbg;           // tuning only: bit 0 = stream planes without computing levels
     double alpha, beta;
+    int split[ST7_MAX_GRID + 1];   // CTA b owns work items [split[b], split[b+1]) (host cost model)
 };
 
 constexpr int ST7_RING_MAX = 12;
@@ -197,11 +207,20 @@ __device__ __forceinline__ void st7_level(const Blk<float, VY>& ZM, const Blk<fl
         if (EXACT) {   // oracle order (X2)
             sa = __fadd2_rn(__fadd2_rn(sxa, __fadd2_rn(yma, ypa)), __fadd2_rn(ZM.a[j], ZP.a[j]));
             sb = __fadd2_rn(__fadd2_rn(sxb, __fadd2_rn(ymb, ypb)), __fadd2_rn(ZM.b[j], ZP.b[j]));
+        } else if (ST_ZLAST) {
+            // tolerance build: the z+1 plane (produced by the previous level in this
+            // same round) enters last, by FMA, so consecutive levels overlap:
+            // R = beta*zp + (alpha*c + beta*((y + x) + zm)) -- still 7 packed ops
+            sa = __fadd2_rn(__fadd2_rn(__fadd2_rn(yma, ypa), sxa), ZM.a[j]);
+            sb = __fadd2_rn(__fadd2_rn(__fadd2_rn(ymb, ypb), sxb), ZM.b[j]);
         } else {       // shuffled X terms last: the y/z sums overlap the shuffle latency
             sa = __fadd2_rn(__fadd2_rn(__fadd2_rn(yma, ypa), __fadd2_rn(ZM.a[j], ZP.a[j])), sxa);
             sb = __fadd2_rn(__fadd2_rn(__fadd2_rn(ymb, ypb), __fadd2_rn(ZM.b[j], ZP.b[j])), sxb);
         }
-        if (EXACT) {
+        if (!EXACT && ST_ZLAST) {
+            R.a[j] = __ffma2_rn(k.beA, ZP.a[j], __ffma2_rn(k.alA, C.a[j], __fmul2_rn(k.beA, sa)));
+            R.b[j] = __ffma2_rn(k.beB, ZP.b[j], __ffma2_rn(k.alB, C.b[j], __fmul2_rn(k.beB, sb)));
+        } else if (EXACT) {
             R.a[j] = make_float2(__fadd_rn(__fmul_rn(k.alA.x, C.a[j].x), __fmul_rn(k.beA.x, sa.x)),
                                  __fadd_rn(__fmul_rn(k.alA.y, C.a[j].y), __fmul_rn(k.beA.y, sa.y)));
             R.b[j] = make_float2(__fadd_rn(__fmul_rn(k.alB.x, C.b[j].x), __fmul_rn(k.beB.x, sb.x)),
@@ -232,7 +251,13 @@ __device__ __forceinline__ void st7_level(const Blk<double, VY>& ZM, const Blk<d
             const double c = C.v[j][i];
             const double xm = i == 0 ? left : C.v[j][0], xp = i == 1 ? right : C.v[j][1];
             const double ym = j > 0 ? C.v[j - 1][i] : top.v[i], yp = j < VY - 1 ? C.v[j + 1][i] : bot.v[i];
-            const double sx = __dadd_rn(xm, xp), sy = __dadd_rn(ym, yp), sz = __dadd_rn(ZM.v[j][i], ZP.v[j][i]);
+            const double sx = __dadd_rn(xm, xp), sy = __dadd_rn(ym, yp);
+            if (!EXACT && ST_ZLAST) {   // z+1 term last (see the FP32 form)
+                const double s = __dadd_rn(__dadd_rn(sy, sx), ZM.v[j][i]);
+                R.v[j][i] = __fma_rn(k.be[i], ZP.v[j][i], __fma_rn(k.al[i], c, __dmul_rn(k.be[i], s)));
+                continue;
+            }
+            const double sz = __dadd_rn(ZM.v[j][i], ZP.v[j][i]);
             const double s = __dadd_rn(__dadd_rn(sx, sy), sz);
             R.v[j][i] = EXACT ? __dadd_rn(__dmul_rn(k.al[i], c), __dmul_rn(k.be[i], s))
                               : __fma_rn(k.al[i], c, __dmul_rn(k.be[i], s));
@@ -277,7 +302,8 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
 
     // zero the ring once: a boundary plane is formed as 1*c + 0*s and may read a
     // never-loaded neighbour plane slot, which must hold finite values
-    for (int i = tid; i < RING * slot_elems; i += blockDim.x) ring[i] = T(0);
+    for (int i = tid; i < RING * slot_elems * (int)sizeof(T) / 16; i += blockDim.x)
+        reinterpret_cast<float4*>(ring)[i] = make_float4(0.f, 0.f, 0.f, 0.f);
     fence_proxy_async();   // generic-proxy writes before the first TMA (async proxy) writes
     if (tid == 0) {
         prefetch_tensormap(&tmap);
@@ -296,9 +322,8 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
         for (int k = 0; k < 3; ++k) pl[l][k] = B{};   // finite (see Coef)
 
     const int nzo = p.zb - p.za;
-    const long long G = gridDim.x;
-    long long item = p.work * (long long)blockIdx.x / G;
-    const long long item_end = p.work * ((long long)blockIdx.x + 1) / G;
+    long long item = p.split[blockIdx.x];
+    const long long item_end = p.split[blockIdx.x + 1];
     const int zmin = max(0, -p.zbase);
     const int zmax = min(p.nzb - 1, p.nzg - 1 - p.zbase);
     const uint32_t tile_bytes = (uint32_t)(slot_elems * sizeof(T));
@@ -314,19 +339,36 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
     T* outp = reinterpret_cast<T*>(p.out);
     const size_t plane = (size_t)p.nx * p.ny;
 
+    // segment = the part of this CTA's work range inside one tile: planes [za, zb)
+    // of the output, level-0 planes [rl0, rl1] loaded at box corner (Lx, Ly)
+    struct Seg { int tile, za, zb, Lx, Ly, rl0, rl1; };
+    auto seg_at = [&](long long it) {
+        Seg g;
+        g.tile = (int)(it / nzo);
+        const long long seg_end = min(item_end, (long long)(g.tile + 1) * nzo);
+        g.za = p.za + (int)(it - (long long)g.tile * nzo);
+        g.zb = p.za + (int)(seg_end - (long long)g.tile * nzo);
+        g.Lx = (g.tile % p.tiles_x) * p.wx - p.hx;
+        g.Ly = (g.tile / p.tiles_x) * p.wy - D;
+        g.rl0 = max(g.za - D, zmin);
+        g.rl1 = min(g.zb - 1 + D, zmax);
+        return g;
+    };
+    int pre = 0;   // loads of the NEXT segment issued during this one's epilog (thread 0 only)
+
     while (item < item_end) {
-        const int tile = (int)(item / nzo);
-        const long long tile_end = (long long)(tile + 1) * nzo;
-        const long long seg_end = min(item_end, tile_end);
-        const int za = p.za + (int)(item - (long long)tile * nzo);
-        const int zb = p.za + (int)(seg_end - (long long)tile * nzo);
-        item = seg_end;
+        const Seg sg = seg_at(item);
+        const int tile = sg.tile, za = sg.za, zb = sg.zb;
+        item += zb - za;
+        // the next segment's first planes are loaded while this one drains
+        const bool has_next = item < item_end;
+        const Seg nx = seg_at(has_next ? item : item - 1);
 
         const int ix = tile % p.tiles_x, iy = tile / p.tiles_x;
         const int ox0 = ix * p.wx, ox1 = min(ox0 + p.wx, p.nx);
         const int oy0 = iy * p.wy, oy1 = min(oy0 + p.wy, p.ny);
-        const int Lx = ox0 - p.hx;
-        const int Ly = oy0 - D;
+        const int Lx = sg.Lx;
+        const int Ly = sg.Ly;
         const int xg0 = Lx + VX * tx;
         uint32_t xfix = 0, rowfix = 0, rowmask = 0;
 #pragma unroll
@@ -345,20 +387,21 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
 
         // level-0 planes to load, rounds, and the steady rounds (every level
         // active, no z-shell plane): those run without any per-level check
-        const int rl0 = max(za - D, zmin);
-        const int rl1 = min(zb - 1 + D, zmax);
+        const int rl0 = sg.rl0;
+        const int rl1 = sg.rl1;
         const int r0 = rl0;
         const int r1 = zb - 1 + D;
         const int rs0 = max(max(za + D, zmin + D), -p.zbase + D + 1);
         const int rs1 = min(min(zb - 1 + D, zmax + 1), min(rl1, p.nzg - 1 - p.zbase));
         const uint32_t kbase = nload;
         if (tid == 0) {
-            for (int q = rl0; q <= min(rl0 + PF - 1, rl1); ++q) {
+            for (int q = rl0 + pre; q <= min(rl0 + PF - 1, rl1); ++q) {
                 const uint32_t k = kbase + (q - rl0);
                 uint64_t* bar = &bars[k % RING];
                 mbar_arrive_expect_tx(bar, tile_bytes);
                 tma_load_3d(ring + (k % RING) * slot_elems, &tmap, bar, Lx, Ly, q);
             }
+            pre = 0;
         }
         nload = kbase + (uint32_t)max(0, rl1 - rl0 + 1);
         // ring slot / parity of plane q, tracked incrementally (no division in the loop)
@@ -373,12 +416,25 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
         auto round = [&](auto PHc, auto STEADYc, int r) {
             constexpr int PH = decltype(PHc)::value;
             constexpr bool STEADY = decltype(STEADYc)::value;
+            // (a copy of the round loop without the per-level y-shell branch for
+            // warps with no shell row was measured 25% SLOWER: the branch keeps
+            // ptxas from interleaving levels, which costs registers and moves)
+            const bool ysl = yslow;
             constexpr int PREV = PH % 3, CUR = (PH + 1) % 3, NEW = (PH + 2) % 3;
             // issue the load of plane r + PF (its slot was freed by the barrier that ended round r-1)
-            if (tid == 0 && r + PF <= rl1) {
-                uint64_t* bar = &bars[slot_f];
-                mbar_arrive_expect_tx(bar, tile_bytes);
-                tma_load_3d(ring + slot_f * slot_elems, &tmap, bar, Lx, Ly, r + PF);
+            if (tid == 0) {
+                if (r + PF <= rl1) {
+                    uint64_t* bar = &bars[slot_f];
+                    mbar_arrive_expect_tx(bar, tile_bytes);
+                    tma_load_3d(ring + slot_f * slot_elems, &tmap, bar, Lx, Ly, r + PF);
+                } else if (has_next && pre < PF && pre == r + PF - rl1 - 1 && nx.rl0 + pre <= nx.rl1) {
+                    // slot_f holds ring sequence number kbase + (r + PF - rl0), which is the
+                    // next segment's plane rl0' + pre (pre = r + PF - rl1 - 1): free since round r-1
+                    uint64_t* bar = &bars[slot_f];
+                    mbar_arrive_expect_tx(bar, tile_bytes);
+                    tma_load_3d(ring + slot_f * slot_elems, &tmap, bar, nx.Lx, nx.Ly, nx.rl0 + pre);
+                    ++pre;
+                }
             }
             // level 0: plane r has landed in the ring
             if (STEADY || r <= rl1) mbar_wait(&bars[slot_r], par_r);
@@ -393,7 +449,7 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                 Row<T> tnn, bnn;
     #pragma unroll
                 for (int l = 1; l <= D; ++l) {
-                    if (p.dbg & 1) break;   // tuning only: stream the planes without computing
+                    if (ST7_DBG && (p.dbg & 1)) break;   // tuning build only: stream the planes without computing
                     const int z = r - l;
                     const int zpar = rpar ^ (l & 1);
                     const XN<T, VY> xnl = xnn;
@@ -427,17 +483,17 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                         }
                         const XN<T, VY> xc = xshuf<NTX, VY>(c);
                         if (!STEADY && zfix)
-                            st7_level<NTX, VY, EXACT>(zm, c, zp, xc, top, bot, Coef<T>::fixed(), yslow, rowfix, dst);
+                            st7_level<NTX, VY, EXACT>(zm, c, zp, xc, top, bot, Coef<T>::fixed(), ysl, rowfix, dst);
                         else
-                            st7_level<NTX, VY, EXACT>(zm, c, zp, xc, top, bot, kc, yslow, rowfix, dst);
+                            st7_level<NTX, VY, EXACT>(zm, c, zp, xc, top, bot, kc, ysl, rowfix, dst);
                     } else {
                         const int lp = l > 1 ? l - 1 : 1;
                         if (!STEADY && zfix)
                             st7_level<NTX, VY, EXACT>(pl[lp][PREV], pl[lp][CUR], pl[lp][NEW], xnl, tl, bl,
-                                                      Coef<T>::fixed(), yslow, rowfix, dst);
+                                                      Coef<T>::fixed(), ysl, rowfix, dst);
                         else
                             st7_level<NTX, VY, EXACT>(pl[lp][PREV], pl[lp][CUR], pl[lp][NEW], xnl, tl, bl, kc,
-                                                      yslow, rowfix, dst);
+                                                      ysl, rowfix, dst);
                     }
                     if (l < D) {
                         V* xb = xw + ((l - 1) * 4 + zpar * 2) * MAXT;
@@ -453,7 +509,7 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                 // levels 1..D: level l computes plane z = r - l
     #pragma unroll
                 for (int l = 1; l <= D; ++l) {
-                    if (p.dbg & 1) break;   // tuning only: stream the planes without computing
+                    if (ST7_DBG && (p.dbg & 1)) break;   // tuning build only: stream the planes without computing
                     const int z = r - l;
                     bool zfix = false;
                     if (!STEADY) {
@@ -486,17 +542,17 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                             zp.load_nat(j, s0 + j * TX);
                         }
                         if (!STEADY && zfix)
-                            st7_level<NTX, VY, EXACT>(zm, c, zp, top, bot, Coef<T>::fixed(), yslow, rowfix, dst);
+                            st7_level<NTX, VY, EXACT>(zm, c, zp, top, bot, Coef<T>::fixed(), ysl, rowfix, dst);
                         else
-                            st7_level<NTX, VY, EXACT>(zm, c, zp, top, bot, kc, yslow, rowfix, dst);
+                            st7_level<NTX, VY, EXACT>(zm, c, zp, top, bot, kc, ysl, rowfix, dst);
                     } else {
                         const int lp = l > 1 ? l - 1 : 1;
                         if (!STEADY && zfix)
                             st7_level<NTX, VY, EXACT>(pl[lp][PREV], pl[lp][CUR], pl[lp][NEW], top, bot,
-                                                      Coef<T>::fixed(), yslow, rowfix, dst);
+                                                      Coef<T>::fixed(), ysl, rowfix, dst);
                         else
                             st7_level<NTX, VY, EXACT>(pl[lp][PREV], pl[lp][CUR], pl[lp][NEW], top, bot, kc,
-                                                      yslow, rowfix, dst);
+                                                      ysl, rowfix, dst);
                     }
                     if (l < D) {
                         V* xb = xw + ((l - 1) * 4 + zpar * 2) * MAXT;

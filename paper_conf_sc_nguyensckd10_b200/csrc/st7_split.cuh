@@ -54,9 +54,8 @@ st7_35d_split_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p
     __syncthreads();
 
     const int nzo = p.zb - p.za;
-    const long long G = gridDim.x;
-    const long long item0 = p.work * (long long)blockIdx.x / G;
-    const long long item_end = p.work * ((long long)blockIdx.x + 1) / G;
+    const long long item0 = p.split[blockIdx.x];
+    const long long item_end = p.split[blockIdx.x + 1];
     const int zmin = max(0, -p.zbase);
     const int zmax = min(p.nzb - 1, p.nzg - 1 - p.zbase);
     const uint32_t tile_bytes = (uint32_t)(slot_elems * sizeof(T));
