@@ -431,8 +431,24 @@ static int launch7(st_plan* p, const void* src, void* dst, int d, double alpha, 
     if (prm.work <= 0) return ST_OK;
     const int grid = std::min(sv.grid_cap > 0 ? std::min(g->grid, sv.grid_cap) : g->grid, ST7_MAX_GRID);
     split_work(prm.ntiles, sv.zb - sv.za, d, grid, prm.split);
+    // tuning builds (-DST7_PROF=1): ST_PROF_OUT=file appends per-warp phase clocks of every launch
+    const char* prof_out = getenv("ST_PROF_OUT");
+    const size_t prof_n = (size_t)grid * 16 * 8;
+    if (prof_out && cudaMalloc(&prm.prof, prof_n * 8) == cudaSuccess) cudaMemset(prm.prof, 0, prof_n * 8);
     cudaError_t e = g->fn(&map, prm, grid, g->threads, g->smem, sv.stream ? sv.stream : p->stream);
     if (e != cudaSuccess) return fail(ST_ECUDA, "st7 launch (d=%d): %s", d, cudaGetErrorString(e));
+    if (prm.prof) {
+        std::vector<unsigned long long> h(prof_n);
+        cudaStreamSynchronize(sv.stream ? sv.stream : p->stream);
+        cudaMemcpy(h.data(), prm.prof, prof_n * 8, cudaMemcpyDeviceToHost);
+        cudaFree(prm.prof);
+        if (FILE* f = fopen(prof_out, "ab")) {
+            const int hdr[4] = {grid, g->maxt / 32, d, (int)(sv.zb - sv.za)};
+            fwrite(hdr, sizeof hdr, 1, f);
+            fwrite(h.data(), 8, prof_n, f);
+            fclose(f);
+        }
+    }
     ++p->launches;
     return ST_OK;
 }

@@ -34,6 +34,15 @@
 #ifndef ST7_DBG
 #define ST7_DBG 0
 #endif
+#ifndef ST7_L0REG
+#define ST7_L0REG 1
+#endif
+#ifndef ST7_LOOKAHEAD
+#define ST7_LOOKAHEAD 0
+#endif
+#ifndef ST7_PROF
+#define ST7_PROF 0
+#endif
 
 namespace st35d {
 
@@ -54,6 +63,7 @@ struct St7Params {
     int dbg;           // tuning only: bit 0 = stream planes without computing levels
     double alpha, beta;
     int split[ST7_MAX_GRID + 1];   // CTA b owns work items [split[b], split[b+1]) (host cost model)
+    unsigned long long* prof;      // ST7_PROF builds only: per-warp phase clocks [cta][warp][8]
 };
 
 constexpr int ST7_RING_MAX = 12;
@@ -293,7 +303,11 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
     const int TY = NTY * VY;
     const T al = T(p.alpha), be = T(p.beta);
 
-    const int RING = p.ring, PF = p.ring - 3;   // ring keeps planes r-2, r-1, r for level 1
+    // the ring keeps the level-0 planes level 1 reads at round r: r-1 (its Y
+    // neighbour rows) and r (ST7_L0REG: the Z window of level 0 is in registers),
+    // or r-2, r-1, r (level 1 reads all three planes from shared memory)
+    constexpr int KEEP = ST7_L0REG ? 2 : 3;
+    const int RING = p.ring, PF = p.ring - KEEP;
     T* ring = reinterpret_cast<T*>(smem_raw);                      // [RING][TY][TX]
     const int slot_elems = TX * TY;
     // row exchange buffer [level 1..D-1][parity][N row / S row][MAXT] (16-byte rows)
@@ -314,10 +328,12 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
 
     // register planes: level l (1..D-1), rotating slot (prev / cur / new); level 0
     // is read straight from the TMA ring (index 0 unused)
+    unsigned long long pr_t0 = ST7_PROF ? clock64() : 0, pr_wait = 0, pr_comp = 0, pr_bar = 0, pr_nr = 0, pr_ns = 0,
+                       pr_ta = 0;
     B pl[D][3];
     B outv;
 #pragma unroll
-    for (int l = 1; l < D; ++l)
+    for (int l = 0; l < D; ++l)
 #pragma unroll
         for (int k = 0; k < 3; ++k) pl[l][k] = B{};   // finite (see Coef)
 
@@ -356,7 +372,9 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
     };
     int pre = 0;   // loads of the NEXT segment issued during this one's epilog (thread 0 only)
 
+    unsigned long long pr_seg = 0, pr_first = 0;
     while (item < item_end) {
+        const unsigned long long pr_ts = ST7_PROF ? clock64() : 0;
         const Seg sg = seg_at(item);
         const int tile = sg.tile, za = sg.za, zb = sg.zb;
         item += zb - za;
@@ -437,11 +455,19 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                 }
             }
             // level 0: plane r has landed in the ring
+            if (ST7_PROF) pr_ta = clock64();
             if (STEADY || r <= rl1) mbar_wait(&bars[slot_r], par_r);
+            unsigned long long pr_tb = 0;
+            if (ST7_PROF) { pr_tb = clock64(); pr_wait += pr_tb - pr_ta; ++pr_nr; pr_ns += STEADY; }
             const int rpar = r & 1;
+            if (ST7_L0REG && (STEADY || r <= rl1)) {   // level 0, plane r: my rows into the register Z window
+                const T* s0 = ring + slot_r * slot_elems + my_off;
+    #pragma unroll
+                for (int j = 0; j < VY; ++j) pl[0][NEW].load_nat(j, s0 + j * TX);
+            }
             // (The look-ahead exchange is measured faster for FP64 and VY = 2; the
             // FP32 VY = 4 blocks have no registers to spare and exchange per level.)
-            if constexpr (sizeof(T) == 8 || VY == 2) {
+            if constexpr (sizeof(T) == 8 || VY == 2 || ST7_LOOKAHEAD) {
                 // levels 1..D: level l computes plane z = r - l.  The X-neighbour
                 // shuffles and exchange-row loads of level l+1 (whose centre plane
                 // pl[l][CUR] exists since round r-1) are issued before level l computes.
@@ -468,18 +494,22 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                         zfix = (zg == 0) || (zg == p.nzg - 1);
                     }
                     B& dst = l < D ? pl[l < D ? l : 1][NEW] : outv;
-                    if (l == 1) {   // level-0 planes r-2, r-1, r of my block straight from the TMA ring
+                    if (l == 1) {   // level-0 planes r-2, r-1, r of my block
                         const T* sl = ring + slot_m1 * slot_elems;   // level-0 neighbour rows of plane r-1
                         const Row<T> top = row_nat(sl + top_off), bot = row_nat(sl + bot_off);
                         B zm, c, zp;
-                        const T* s2 = ring + slot_m2 * slot_elems + my_off;
-                        const T* s1 = ring + slot_m1 * slot_elems + my_off;
-                        const T* s0 = ring + slot_r * slot_elems + my_off;
+                        if (ST7_L0REG) {
+                            zm = pl[0][PREV]; c = pl[0][CUR]; zp = pl[0][NEW];
+                        } else {
+                            const T* s2 = ring + slot_m2 * slot_elems + my_off;
+                            const T* s1 = ring + slot_m1 * slot_elems + my_off;
+                            const T* s0 = ring + slot_r * slot_elems + my_off;
     #pragma unroll
-                        for (int j = 0; j < VY; ++j) {
-                            zm.load_nat(j, s2 + j * TX);
-                            c.load_nat(j, s1 + j * TX);
-                            zp.load_nat(j, s0 + j * TX);
+                            for (int j = 0; j < VY; ++j) {
+                                zm.load_nat(j, s2 + j * TX);
+                                c.load_nat(j, s1 + j * TX);
+                                zp.load_nat(j, s0 + j * TX);
+                            }
                         }
                         const XN<T, VY> xc = xshuf<NTX, VY>(c);
                         if (!STEADY && zfix)
@@ -530,16 +560,20 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                         bot = row_x(xbot + o);
                     }
                     B& dst = l < D ? pl[l < D ? l : 1][NEW] : outv;
-                    if (l == 1) {   // level-0 planes r-2, r-1, r of my block straight from the ring
+                    if (l == 1) {   // level-0 planes r-2, r-1, r of my block
                         B zm, c, zp;
-                        const T* s2 = ring + slot_m2 * slot_elems + my_off;
-                        const T* s1 = ring + slot_m1 * slot_elems + my_off;
-                        const T* s0 = ring + slot_r * slot_elems + my_off;
+                        if (ST7_L0REG) {
+                            zm = pl[0][PREV]; c = pl[0][CUR]; zp = pl[0][NEW];
+                        } else {
+                            const T* s2 = ring + slot_m2 * slot_elems + my_off;
+                            const T* s1 = ring + slot_m1 * slot_elems + my_off;
+                            const T* s0 = ring + slot_r * slot_elems + my_off;
     #pragma unroll
-                        for (int j = 0; j < VY; ++j) {
-                            zm.load_nat(j, s2 + j * TX);
-                            c.load_nat(j, s1 + j * TX);
-                            zp.load_nat(j, s0 + j * TX);
+                            for (int j = 0; j < VY; ++j) {
+                                zm.load_nat(j, s2 + j * TX);
+                                c.load_nat(j, s1 + j * TX);
+                                zp.load_nat(j, s0 + j * TX);
+                            }
                         }
                         if (!STEADY && zfix)
                             st7_level<NTX, VY, EXACT>(zm, c, zp, top, bot, Coef<T>::fixed(), ysl, rowfix, dst);
@@ -565,7 +599,10 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                     }
                 }
             }
+            unsigned long long pr_tc = 0;
+            if (ST7_PROF) { pr_tc = clock64(); pr_comp += pr_tc - pr_tb; }
             __syncthreads();
+            if (ST7_PROF) pr_bar += clock64() - pr_tc;
             pout += plane;
             // advance the ring cursors
             slot_m2 = slot_m1;
@@ -578,6 +615,7 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
             else round(PHc, std::false_type{}, r);
         };
 
+        if (ST7_PROF) { const unsigned long long t = clock64(); pr_seg += t - pr_ts; if (!pr_first) pr_first = t - pr_t0; }
         for (int r = r0; r <= r1;) {
             any_round(std::integral_constant<int, 0>{}, r);
             if (++r > r1) break;
@@ -586,6 +624,11 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
             any_round(std::integral_constant<int, 2>{}, r);
             ++r;
         }
+    }
+    if (ST7_PROF && p.prof && (tid & 31) == 0) {
+        unsigned long long* o = p.prof + ((size_t)blockIdx.x * (MAXT / 32) + tid / 32) * 8;
+        o[0] = clock64() - pr_t0; o[1] = pr_wait; o[2] = pr_comp; o[3] = pr_bar; o[4] = pr_nr; o[5] = pr_ns;
+        o[6] = pr_seg; o[7] = pr_first;
     }
 }
 
