@@ -791,8 +791,11 @@ static int launch_lbm(st_plan* p, const void* src, void* dst, const uint8_t* fla
     else lid_coeffs<double>(p->lid, prm.lidc);
     const long long cells = (long long)(sv.zb - sv.za) * p->nx * p->ny;
     if (cells <= 0) return ST_OK;
-    const int grid = (int)std::min<long long>((cells + 255) / 256, (long long)p->sms * (p->dtype == ST_F32 ? 4 : 3));
-    cudaError_t e = lbm_push_launch(p->dtype == ST_F32 ? 0 : 1, p->exact, src, dst, flags, prm, grid,
+    // one wave of resident 256-thread CTAs (launch bounds: 4 per SM FP32, 2 FP64), grid-stride over the cells
+    int bps = p->dtype == ST_F32 ? 4 : 2;
+    if (const char* e = getenv("ST_LBM_BPS")) bps = std::max(1, atoi(e));   // A/B tuning
+    const int grid = (int)std::min<long long>((cells + 255) / 256, (long long)p->sms * bps);
+    cudaError_t e = lbm_push_launch(p->dtype == ST_F32 ? 0 : 1, p->exact, src, dst, sv.fl2, prm, grid,
                                     sv.stream ? sv.stream : p->stream);
     if (e != cudaSuccess) return fail(ST_ECUDA, "lbm launch: %s", cudaGetErrorString(e));
     ++p->launches;
@@ -825,7 +828,7 @@ static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T
     // the on-chip multi-level sweep lbm_35d (ST_LBM_35D=1 forces it for dim_T = 1)
     const bool push = max_lbm_depth(p) == 1 && getenv("ST_LBM_35D") == nullptr && p->dist.mode == Dist::SINGLE;
     // neighbour-flag prepass, every call (a reused flags pointer may hold new contents; ~1 pass over the flags)
-    if (!push && p->dist.mode != Dist::LOOPBACK) {
+    if (p->dist.mode != Dist::LOOPBACK) {
         const size_t cells = (size_t)p->nx * p->ny * p->dist.nzb;
         if (p->fl2_bytes < cells) {
             if (p->fl2) cudaFree(p->fl2);

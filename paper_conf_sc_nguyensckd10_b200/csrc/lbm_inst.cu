@@ -4,18 +4,18 @@
 namespace st35d {
 
 template <typename T, bool E>
-static cudaError_t push_t(const void* src, void* dst, const uint8_t* flags, const LbmParams& p, int grid,
+static cudaError_t push_t(const void* src, void* dst, const uint8_t* fl2, const LbmParams& p, int grid,
                           cudaStream_t s) {
-    lbm_push_kernel<T, E><<<grid, 256, 0, s>>>(static_cast<const T*>(src), static_cast<T*>(dst), flags, p);
+    lbm_push_kernel<T, E><<<grid, 256, 0, s>>>(static_cast<const T*>(src), static_cast<T*>(dst), fl2, p);
     return cudaGetLastError();
 }
 
-cudaError_t lbm_push_launch(int dtype, bool exact, const void* src, void* dst, const uint8_t* flags,
+// fl2 = the lbm_fl2 prepass output of the flags
+cudaError_t lbm_push_launch(int dtype, bool exact, const void* src, void* dst, const uint8_t* fl2,
                             const LbmParams& p, int grid, cudaStream_t s) {
-    if (dtype == 0) return exact ? push_t<float, true>(src, dst, flags, p, grid, s)
-                                 : push_t<float, false>(src, dst, flags, p, grid, s);
-    return exact ? push_t<double, true>(src, dst, flags, p, grid, s)
-                 : push_t<double, false>(src, dst, flags, p, grid, s);
+    if (dtype == 0) return exact ? push_t<float, true>(src, dst, fl2, p, grid, s)
+                                 : push_t<float, false>(src, dst, fl2, p, grid, s);
+    return exact ? push_t<double, true>(src, dst, fl2, p, grid, s) : push_t<double, false>(src, dst, fl2, p, grid, s);
 }
 
 template <typename T, int D, bool E>

@@ -17,6 +17,7 @@
 #pragma once
 #include "common.cuh"
 
+
 namespace st35d {
 
 struct LbmParams {
@@ -125,42 +126,61 @@ __device__ __forceinline__ void collide(T (&f)[19], T omega) {
 }
 
 // dim_T = 1: push form, one thread per cell, grid-stride over the updated planes.
+// fl2 = flags | 0x80 for FLUID cells with a non-FLUID neighbour (lbm_fl2 prepass).
+// Every store is predicated on the target cell's flag (WALL / LID links bounce
+// back).  Measured on B200 (256^3 cavity, tools/lbm_ab.sh): an unconditional
+// store path for interior cells is 20-35% SLOWER than flag-gated stores for
+// FP32 — the gating paces the 19 stores of a cell behind short L1 hits instead
+// of bursting them into the LSU queue ahead of other warps' loads — while
+// FP64 (twice the bytes per store) prefers all 18 neighbour flags loaded up
+// front (one round trip), 17.0 vs 15.7 GLUPS.
 template <typename T, bool E>
-__global__ void __launch_bounds__(256, (sizeof(T) == 4 ? 4 : 3))
-lbm_push_kernel(const T* __restrict__ src, T* __restrict__ dst, const uint8_t* __restrict__ flags,
+__global__ void __launch_bounds__(256, (sizeof(T) == 4 ? 4 : 2))
+lbm_push_kernel(const T* __restrict__ src, T* __restrict__ dst, const uint8_t* __restrict__ fl2,
                 const LbmParams p) {
+    constexpr bool BATCH = sizeof(T) == 8;
     const size_t plane = (size_t)p.nx * p.ny;
     const size_t nc = plane * p.nzb;              // SoA stride of one population
     const size_t c0 = (size_t)p.za * plane;
     const size_t ncell = (size_t)(p.zb - p.za) * plane;
     const T omega = T(p.omega);
+    const int nx = p.nx;
     for (size_t t = blockIdx.x * (size_t)blockDim.x + threadIdx.x; t < ncell; t += (size_t)gridDim.x * blockDim.x) {
         const size_t c = c0 + t;
-        const uint8_t fl = flags[c];
+        const uint32_t fl = fl2[c];
+        const T* __restrict__ s = src + c;
         T f[19];
 #pragma unroll
-        for (int i = 0; i < 19; ++i) f[i] = src[i * nc + c];
-        if (fl != 0) {
+        for (int i = 0; i < 19; ++i) f[i] = s[i * nc];
+        T* __restrict__ d = dst + c;
+        if (fl & 0x7fu) {   // WALL / LID: copied through
 #pragma unroll
-            for (int i = 0; i < 19; ++i) dst[i * nc + c] = f[i];
+            for (int i = 0; i < 19; ++i) d[i * nc] = f[i];
             continue;
         }
         collide<T, E>(f, omega);
-        const int nx = p.nx;
+        uint32_t tfl[19];
+        if constexpr (BATCH) {
+            auto ld = [&](auto Ic) {
+                constexpr int I = decltype(Ic)::value;
+                const long long off = (long long)D3Q19<I>::ex + (long long)D3Q19<I>::ey * nx +
+                                      (long long)D3Q19<I>::ez * (long long)plane;
+                tfl[I] = I == 0 ? 0u : (uint32_t)__ldg(fl2 + (size_t)((long long)c + off));
+            };
+            [&]<int... Is>(std::integer_sequence<int, Is...>) { (ld(std::integral_constant<int, Is>{}), ...); }
+            (std::make_integer_sequence<int, 19>{});
+        }
         auto push = [&](auto Ic) {
             constexpr int I = decltype(Ic)::value;
-            constexpr long long off_c = 0;
-            (void)off_c;
             const long long off = (long long)D3Q19<I>::ex + (long long)D3Q19<I>::ey * nx +
                                   (long long)D3Q19<I>::ez * (long long)plane;
-            const size_t tc = (size_t)((long long)c + off);
             if constexpr (I == 0) {
-                dst[c] = f[0];
+                d[0] = f[0];
             } else {
-                const uint8_t tf = flags[tc];
-                if (tf == 0) dst[I * nc + tc] = f[I];
-                else if (tf == 1) dst[D3Q19<I>::opp * nc + c] = f[I];
-                else dst[D3Q19<I>::opp * nc + c] = Ar<T, E>::sub(f[I], T(p.lidc[I]));
+                const uint32_t tf = (BATCH ? tfl[I] : (uint32_t)fl2[(size_t)((long long)c + off)]) & 0x7fu;
+                if (tf == 0) d[I * nc + off] = f[I];
+                else if (tf == 1) d[D3Q19<I>::opp * nc] = f[I];
+                else d[D3Q19<I>::opp * nc] = Ar<T, E>::sub(f[I], T(p.lidc[I]));
             }
         };
         [&]<int... Is>(std::integer_sequence<int, Is...>) { (push(std::integral_constant<int, Is>{}), ...); }
