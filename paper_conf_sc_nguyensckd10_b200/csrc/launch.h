@@ -1,12 +1,32 @@
 // launch.h — internal dispatch between the C-ABI (api.cu) and the kernel
 // instantiation units (st7_inst.cu compiled per dtype/mode, lbm_inst.cu).
 #pragma once
+#include <cstdlib>
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include "st7_kernel.cuh"
 #include "lbm_kernel.cuh"
 
 namespace st35d {
+
+// launch with programmatic stream serialization (PDL): the kernel's prologue may
+// overlap the previous kernel in the stream; the kernel orders its memory
+// accesses after it with griddepcontrol.wait (ST_NO_PDL=1: plain launch, A/B)
+template <typename K, typename... A>
+inline cudaError_t launch_pdl(K kernel, int grid, int threads, size_t smem, cudaStream_t s, A... args) {
+    static const bool off = getenv("ST_NO_PDL") != nullptr;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(threads);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = off ? 0 : 1;
+    return cudaLaunchKernelEx(&cfg, kernel, args...);
+}
 
 using St7LaunchFn = cudaError_t (*)(const CUtensorMap* map, const St7Params& p, int grid, int threads,
                                     size_t smem, cudaStream_t s);

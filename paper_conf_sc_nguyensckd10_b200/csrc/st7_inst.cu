@@ -34,8 +34,7 @@ cudaError_t launch(const CUtensorMap* map, const St7Params& p, int grid, int thr
     auto k = st7_35d_kernel<TT, D, NTX, VY, ST_EXACT != 0, MAXT>;
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    k<<<grid, threads, smem, s>>>(*map, p);
-    return cudaGetLastError();
+    return launch_pdl(k, grid, threads, smem, s, *map, p);
 }
 
 template <int VY, int MAXT>

@@ -325,6 +325,10 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
         fence_mbar_init();
     }
     __syncthreads();
+    // PDL: the setup above overlapped the previous sweep's tail; its output
+    // (this sweep's input) and its reads of our output buffer are complete here
+    pdl_trigger();
+    pdl_wait();
 
     // register planes: level l (1..D-1), rotating slot (prev / cur / new); level 0
     // is read straight from the TMA ring (index 0 unused)
