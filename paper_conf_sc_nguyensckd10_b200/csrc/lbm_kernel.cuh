@@ -59,6 +59,10 @@ template <bool E> struct Ar<double, E> {
     static __device__ __forceinline__ double div(double a, double b) { return __ddiv_rn(a, b); }
 };
 
+template <typename T> struct Rcp;
+template <> struct Rcp<float> { static __device__ __forceinline__ float rn(float x) { return __frcp_rn(x); } };
+template <> struct Rcp<double> { static __device__ __forceinline__ double rn(double x) { return __drcp_rn(x); } };
+
 // signed accumulation of e_a * f over the non-zero components, oracle order (X20)
 template <typename T, bool E, int A, int I = 0>
 __device__ __forceinline__ void jsum(const T (&f)[19], T& acc, bool& first) {
@@ -106,7 +110,13 @@ __device__ __forceinline__ void collide(T (&f)[19], T omega) {
         jy = ((f[3] - f[4]) + (f[7] - f[8])) + ((f[10] - f[9]) + ((f[15] - f[16]) + (f[17] - f[18])));
         jz = ((f[5] - f[6]) + (f[11] - f[12])) + ((f[14] - f[13]) + ((f[15] - f[16]) + (f[18] - f[17])));
     }
-    const T ux = A::div(jx, rho), uy = A::div(jy, rho), uz = A::div(jz, rho);
+    T ux, uy, uz;
+    if (E) {   // oracle: three IEEE divisions
+        ux = A::div(jx, rho); uy = A::div(jy, rho); uz = A::div(jz, rho);
+    } else {   // tolerance mode: one correctly rounded reciprocal, three products
+        const T inv = Rcp<T>::rn(rho);
+        ux = jx * inv; uy = jy * inv; uz = jz * inv;
+    }
     T usq = A::add(A::mul(ux, ux), A::mul(uy, uy));
     usq = A::add(usq, A::mul(uz, uz));
     const T usq15 = A::mul(T(1.5), usq);
@@ -134,7 +144,7 @@ __device__ __forceinline__ void collide(T (&f)[19], T omega) {
 // of bursting them into the LSU queue ahead of other warps' loads — while
 // FP64 (twice the bytes per store) prefers all 18 neighbour flags loaded up
 // front (one round trip), 17.0 vs 15.7 GLUPS.
-template <typename T, bool E>
+template <typename T, bool E, typename IX>
 __global__ void __launch_bounds__(256, (sizeof(T) == 4 ? 4 : 2))
 lbm_push_kernel(const T* __restrict__ src, T* __restrict__ dst, const uint8_t* __restrict__ fl2,
                 const LbmParams p) {
@@ -145,17 +155,18 @@ lbm_push_kernel(const T* __restrict__ src, T* __restrict__ dst, const uint8_t* _
     const size_t ncell = (size_t)(p.zb - p.za) * plane;
     const T omega = T(p.omega);
     const int nx = p.nx;
+    const IX ncx = (IX)nc, pl = (IX)plane;   // 32-bit offsets when 19 populations fit (host choice)
     for (size_t t = blockIdx.x * (size_t)blockDim.x + threadIdx.x; t < ncell; t += (size_t)gridDim.x * blockDim.x) {
         const size_t c = c0 + t;
         const uint32_t fl = fl2[c];
         const T* __restrict__ s = src + c;
         T f[19];
 #pragma unroll
-        for (int i = 0; i < 19; ++i) f[i] = s[i * nc];
+        for (int i = 0; i < 19; ++i) f[i] = s[(IX)i * ncx];
         T* __restrict__ d = dst + c;
         if (fl & 0x7fu) {   // WALL / LID: copied through
 #pragma unroll
-            for (int i = 0; i < 19; ++i) d[i * nc] = f[i];
+            for (int i = 0; i < 19; ++i) d[(IX)i * ncx] = f[i];
             continue;
         }
         collide<T, E>(f, omega);
@@ -163,24 +174,22 @@ lbm_push_kernel(const T* __restrict__ src, T* __restrict__ dst, const uint8_t* _
         if constexpr (BATCH) {
             auto ld = [&](auto Ic) {
                 constexpr int I = decltype(Ic)::value;
-                const long long off = (long long)D3Q19<I>::ex + (long long)D3Q19<I>::ey * nx +
-                                      (long long)D3Q19<I>::ez * (long long)plane;
-                tfl[I] = I == 0 ? 0u : (uint32_t)__ldg(fl2 + (size_t)((long long)c + off));
+                const IX off = (IX)D3Q19<I>::ex + (IX)D3Q19<I>::ey * (IX)nx + (IX)D3Q19<I>::ez * pl;
+                tfl[I] = I == 0 ? 0u : (uint32_t)__ldg(fl2 + c + off);
             };
             [&]<int... Is>(std::integer_sequence<int, Is...>) { (ld(std::integral_constant<int, Is>{}), ...); }
             (std::make_integer_sequence<int, 19>{});
         }
         auto push = [&](auto Ic) {
             constexpr int I = decltype(Ic)::value;
-            const long long off = (long long)D3Q19<I>::ex + (long long)D3Q19<I>::ey * nx +
-                                  (long long)D3Q19<I>::ez * (long long)plane;
+            const IX off = (IX)D3Q19<I>::ex + (IX)D3Q19<I>::ey * (IX)nx + (IX)D3Q19<I>::ez * pl;
             if constexpr (I == 0) {
                 d[0] = f[0];
             } else {
-                const uint32_t tf = (BATCH ? tfl[I] : (uint32_t)fl2[(size_t)((long long)c + off)]) & 0x7fu;
-                if (tf == 0) d[I * nc + off] = f[I];
-                else if (tf == 1) d[D3Q19<I>::opp * nc] = f[I];
-                else d[D3Q19<I>::opp * nc] = Ar<T, E>::sub(f[I], T(p.lidc[I]));
+                const uint32_t tf = (BATCH ? tfl[I] : (uint32_t)fl2[c + off]) & 0x7fu;
+                if (tf == 0) d[(IX)I * ncx + off] = f[I];
+                else if (tf == 1) d[(IX)D3Q19<I>::opp * ncx] = f[I];
+                else d[(IX)D3Q19<I>::opp * ncx] = Ar<T, E>::sub(f[I], T(p.lidc[I]));
             }
         };
         [&]<int... Is>(std::integer_sequence<int, Is...>) { (push(std::integral_constant<int, Is>{}), ...); }
