@@ -132,9 +132,14 @@ def run_reference(args, rank, world):
     import stgen
     n = args.n
     a = stgen.grid7(n, n, n, 2, np.float32)
-    Ts = 2  # bounded sample per step: 2 sweeps of the 256^3 grid
-    for _ in range(max(1, args.warmup)):
-        oracle.st7(a, 0.4, 0.1, 1)
+    # one step = the configs[1] run (T sweeps) when the host finishes the whole
+    # --steps/--warmup run in ~2.5 min at that size; else a bounded sample of Ts sweeps
+    t0 = time.perf_counter()
+    oracle.st7(a, 0.4, 0.1, 4)
+    per_sweep = (time.perf_counter() - t0) / 4
+    Ts = int(max(1, min(args.T, 150.0 / (args.steps + args.warmup) / max(per_sweep, 1e-6))))
+    for _ in range(args.warmup):
+        oracle.st7(a, 0.4, 0.1, Ts)
     t0 = time.perf_counter()
     for _ in range(args.steps):
         oracle.st7(a, 0.4, 0.1, Ts)
@@ -147,7 +152,7 @@ def run_reference(args, rank, world):
         "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": round(dt / args.steps * 1e3, 3), "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "f32", "data": "synthetic (splitmix64 U[0,1), seed 2)",
-        "config": {"workload": f"7-point FP32 {n}^3 (configs[1]); each step a bounded sample of T={Ts} sweeps",
+        "config": {"workload": f"7-point FP32 {n}^3 (configs[1]); each step {Ts} of the T={args.T} sweeps",
                    "grid": [n, n, n], "T_sample": Ts},
         "cpu_baseline": {"value": round(v, 2), "unit": "Mupdates/s", "cores": cores, "kind": "oracle",
                          "sample": f"{n}^3 FP32, {Ts} Jacobi sweeps per step, {args.steps} steps"},
@@ -164,10 +169,15 @@ def cpu_baseline_7pt(n):
     t0 = time.perf_counter()
     oracle.st7(a, 0.4, 0.1, 8)
     t1 = (time.perf_counter() - t0) / 8          # per sweep (incl. the oracle's own copies)
-    Ts = int(max(1, min(5000, round(12.0 / max(t1, 1e-4)))))
+    Ts = int(max(1, min(20000, round(12.0 / max(t1, 1e-4)))))
     t0 = time.perf_counter()
     oracle.st7(a, 0.4, 0.1, Ts)
     dt = time.perf_counter() - t0
+    if dt < 6.0:   # the 8-sweep probe is dominated by per-call overhead: rescale once to ~12 s
+        Ts = int(max(1, min(20000, round(Ts * 12.0 / max(dt, 1e-3)))))
+        t0 = time.perf_counter()
+        oracle.st7(a, 0.4, 0.1, Ts)
+        dt = time.perf_counter() - t0
     return {"value": round((n - 2) ** 3 * Ts / dt / 1e6, 2), "unit": "Mupdates/s",
             "cores": oracle.num_threads(), "kind": "oracle",
             "sample": f"7-point FP32 {n}^3, T={Ts} sweeps ({dt:.1f} s), OpenMP over z"}
@@ -347,6 +357,25 @@ def main():
                                  "dim_T": D5, "dim_T_sweep": sw5, "ms_per_step": round(ms5, 3),
                                  "frac_alu": round(ST7_OPS * upd5 / (ms5 / 1e3) / (ops_peak * 1e12), 4),
                                  "info": inf5}
+        # ablation ladder (Fig. 5(b)): no blocking -> 2.5D (dim_T = 1)
+        # -> 3.5D (measured dim_T), same grid and T; plus the eq. (3) model's dim_T seed (f3)
+        xa = torch.from_numpy(stgen.grid7(n, n, n, 2, np.float32)).cuda()
+        ya = torch.empty_like(xa)
+        with st.Plan(n, n, n, torch.float32, 1) as pn:
+            pn.set_stream(stream)
+            pn.set_variant(st.ST_VARIANT_NAIVE)
+            tn, _ = time_steps(lambda: pn.st7(xa, ya, 0.4, 0.1, T), 2, 1)
+        del xa, ya
+        gamma = 8.0 / ST7_OPS                                    # B per FP instruction
+        Gamma = hbm_gbs * 1e9 / (ops_peak * 1e12)                # B200: measured HBM / FP32 lane-instr rate
+        mdl = st.st_blocking_model(227 * 1024, 4, 1, gamma, Gamma, 0, 0)
+        extras["ablation_f32_256"] = {
+            "unit": "Mupdates/s", "naive_no_blocking": round((n - 2) ** 3 * T / (tn / 2 / 1e3) / 1e6, 1),
+            "2.5D_dim_T_1": sweep.get(1), "3.5D": round(value, 1), "dim_T": D,
+            "model": {"gamma_B_per_instr": round(gamma, 3), "Gamma_B_per_instr": round(Gamma, 4),
+                      "eta_eq3": mdl["eta"], "measured_best_dim_T": D,
+                      "note": "eta = ceil(gamma/Gamma) is where the HBM roof meets the FP32 roof; the "
+                              "measured optimum is lower because the kernel is issue/latency-bound"}}
         # LBM D3Q19 cavity 256^3 (configs[2])
         for dtn, dt_np, tdt in (("f32", np.float32, torch.float32), ("f64", np.float64, torch.float64)):
             nl, Tl = 256, 100

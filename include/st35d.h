@@ -122,6 +122,16 @@ int st_plan_set_lbm_lid(st_plan* plan, double ux, double uy, double uz);
 /* 1: bit-exact kernels (no FMA contraction, oracle operation order). */
 int st_plan_set_bitexact(st_plan* plan, int on);
 
+/* Kernel variant of st7_run (default ST_VARIANT_35D, the 3.5D sweep).
+ * ST_VARIANT_NAIVE is the "no blocking" bar of the ablation ladder (PAPER.md
+ * Fig. 5(b)): one Jacobi step per launch, one
+ * thread per point, seven global loads per update, oracle operation order
+ * (bit-identical to the oracle in either build).  Same contract as st7_run
+ * (in is scratch, T = 0 copies); single-process plans only (a distributed
+ * plan returns ST_EUNSUPPORTED at run time).  lbm_d3q19_run ignores it. */
+enum { ST_VARIANT_35D = 0, ST_VARIANT_NAIVE = 1 };
+int st_plan_set_variant(st_plan* plan, int variant);
+
 /* Waits for the plan stream; returns ST_ECUDA for deferred device faults. */
 int st_plan_sync(st_plan* plan);
 

@@ -46,7 +46,7 @@ class st_blocking(ctypes.Structure):
 _lib = None
 
 EXPORTS = ["st_plan_create", "st7_run", "lbm_d3q19_run", "st_destroy", "st_last_error", "st_last_status",
-           "st_plan_set_stream", "st_plan_set_lbm_lid", "st_plan_set_bitexact", "st_plan_sync",
+           "st_plan_set_stream", "st_plan_set_lbm_lid", "st_plan_set_bitexact", "st_plan_set_variant", "st_plan_sync",
            "st_plan_set_dist", "st_plan_set_loopback_slabs", "st_plan_ghost_planes", "st_plan_local_slab",
            "st_plan_get_info", "st_plan_last_launches", "st_blocking_model", "st_fig3_step",
            "st_nccl_unique_id", "st_slab_range"]
@@ -71,6 +71,7 @@ def lib() -> ctypes.CDLL:
         "st_plan_set_stream": ([P, P], I),
         "st_plan_set_lbm_lid": ([P, D, D, D], I),
         "st_plan_set_bitexact": ([P, I], I),
+        "st_plan_set_variant": ([P, I], I),
         "st_plan_sync": ([P], I),
         "st_plan_set_dist": ([P, P, I, I], I),
         "st_plan_set_loopback_slabs": ([P, I], I),
@@ -149,6 +150,14 @@ def st_plan_set_lbm_lid(plan: int, ux: float, uy: float, uz: float) -> int:
 
 def st_plan_set_bitexact(plan: int, on: bool) -> int:
     return _check(lib().st_plan_set_bitexact(plan, 1 if on else 0))
+
+
+ST_VARIANT_35D, ST_VARIANT_NAIVE = 0, 1
+
+
+def st_plan_set_variant(plan: int, variant: int) -> int:
+    """ST_VARIANT_NAIVE: the no-blocking ablation baseline (include/st35d.h)."""
+    return _check(lib().st_plan_set_variant(plan, int(variant)))
 
 
 def st_plan_sync(plan: int) -> int:
@@ -233,6 +242,9 @@ class Plan:
 
     def set_stream(self, stream) -> None:
         st_plan_set_stream(self.h, stream)
+
+    def set_variant(self, variant: int) -> None:
+        st_plan_set_variant(self.h, variant)
 
     def set_bitexact(self, on: bool) -> None:
         st_plan_set_bitexact(self.h, on)

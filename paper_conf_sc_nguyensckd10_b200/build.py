@@ -47,6 +47,7 @@ COMMON = ARCH + ["-O3", "-lineinfo", "-std=c++20", "--expt-relaxed-constexpr", "
 UNITS = [
     ("api.cu", "api.o", []),
     ("lbm_inst.cu", "lbm_inst.o", []),
+    ("naive.cu", "naive.o", []),
     ("model.cpp", "model.o", []),
 ] + [
     ("st7_inst.cu", f"st7_{tn}_{mode}.o", [f"-DST_T={t}", f"-DST_TNAME={tn}", f"-DST_EXACT={ex}"])

@@ -97,6 +97,7 @@ struct st_plan {
     cudaStream_t stream = nullptr;
     bool own_stream = false;
     bool exact = false;
+    int variant = ST_VARIANT_35D;    // st_plan_set_variant (ablation baseline ST_VARIANT_NAIVE)
     double lid[3] = {0.05, 0.0, 0.0};
     int launches = 0;
     // host-pointer staging
@@ -282,6 +283,13 @@ extern "C" int st_plan_set_stream(st_plan* p, void* s) {
 extern "C" int st_plan_set_lbm_lid(st_plan* p, double ux, double uy, double uz) {
     if (!p) return fail(ST_EINVAL, "NULL plan");
     p->lid[0] = ux; p->lid[1] = uy; p->lid[2] = uz;
+    return ST_OK;
+}
+
+extern "C" int st_plan_set_variant(st_plan* p, int variant) {
+    if (!p) return fail(ST_EINVAL, "NULL plan");
+    if (variant != ST_VARIANT_35D && variant != ST_VARIANT_NAIVE) return fail(ST_EINVAL, "variant %d", variant);
+    p->variant = variant;
     return ST_OK;
 }
 
@@ -675,6 +683,21 @@ static int run7_device(st_plan* p, const void* in, void* out, double alpha, doub
     p->launches = 0;
     if (T == 0) {
         CUDA_TRY(cudaMemcpyAsync(out, in, n, cudaMemcpyDeviceToDevice, p->stream));
+        return ST_OK;
+    }
+    if (p->variant == ST_VARIANT_NAIVE) {   // ablation baseline: T single-step launches, ping-pong
+        if (p->dist.mode != Dist::SINGLE) return fail(ST_EUNSUPPORTED, "the naive variant is single-process only");
+        const void* src = in;
+        void* bufs[2] = {const_cast<void*>(in), out};
+        for (int k = 0; k < T; ++k) {
+            void* dst = bufs[(k + 1) % 2];
+            cudaError_t e = st7_naive_launch(p->dtype == ST_F32 ? 0 : 1, src, dst, p->nx, p->ny, p->nz, alpha, beta,
+                                             p->stream);
+            if (e != cudaSuccess) return fail(ST_ECUDA, "naive launch: %s", cudaGetErrorString(e));
+            ++p->launches;
+            src = dst;
+        }
+        if (T % 2 == 0) CUDA_TRY(cudaMemcpyAsync(out, in, n, cudaMemcpyDeviceToDevice, p->stream));
         return ST_OK;
     }
     std::vector<int> ds = sweep_depths(T, p->dimK);

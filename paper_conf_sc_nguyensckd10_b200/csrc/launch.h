@@ -46,6 +46,8 @@ cudaError_t lbm_push_launch(int dtype, bool exact, const void* src, void* dst, c
                             const LbmParams& p, int grid, cudaStream_t s);
 cudaError_t lbm35_launch(int dtype, bool exact, int D, const Lbm35Params& p, int grid, int threads, size_t smem,
                          cudaStream_t s);
+cudaError_t st7_naive_launch(int dtype, const void* in, void* out, int nx, int ny, int nz, double alpha,
+                             double beta, cudaStream_t s);
 cudaError_t lbm_fl2(const uint8_t* flags, uint8_t* fl2, int nx, int ny, int nz, cudaStream_t s);
 constexpr int LBM35_MAX_D = 3;
 cudaError_t lbm_shell_check(const uint8_t* flags, int nx, int ny, int nz, int* d_count, cudaStream_t s);

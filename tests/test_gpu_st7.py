@@ -132,3 +132,21 @@ def test_config3_512_full_grid(oracle_lib):
     assert relerr(got, ref) <= TOL[np.float32]
     got, _ = run_gpu(a, 0.4, 0.1, T, 4, exact=True)
     assert np.array_equal(got, ref)
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+@pytest.mark.parametrize("T", [0, 1, 4, 7])
+def test_naive_variant_bitexact(oracle_lib, dtype, T):
+    # the no-blocking ablation baseline (ST_VARIANT_NAIVE) computes in the oracle's order
+    nx, ny, nz = (68, 52, 37) if dtype == np.float32 else (66, 40, 21)
+    a = stgen.grid7(nx, ny, nz, 7, dtype)
+    ref = oracle_lib.st7(a, 0.4, 0.1, T)
+    dt = torch.float32 if dtype == np.float32 else torch.float64
+    with st.Plan(nx, ny, nz, dt, 1) as p:
+        p.set_variant(st.ST_VARIANT_NAIVE)
+        x = torch.from_numpy(a).cuda()
+        y = torch.empty_like(x)
+        p.st7(x, y, 0.4, 0.1, T)
+        p.sync()
+        assert p.last_launches() == T
+    assert np.array_equal(y.cpu().numpy(), ref)
