@@ -441,7 +441,7 @@ static int launch7(st_plan* p, const void* src, void* dst, int d, double alpha, 
     split_work(prm.ntiles, sv.zb - sv.za, d, grid, prm.split);
     // tuning builds (-DST7_PROF=1): ST_PROF_OUT=file appends per-warp phase clocks of every launch
     const char* prof_out = getenv("ST_PROF_OUT");
-    const size_t prof_n = (size_t)grid * 16 * 8;
+    const size_t prof_n = (size_t)grid * 16 * 10;
     if (prof_out && cudaMalloc(&prm.prof, prof_n * 8) == cudaSuccess) cudaMemset(prm.prof, 0, prof_n * 8);
     cudaError_t e = g->fn(&map, prm, grid, g->threads, g->smem, sv.stream ? sv.stream : p->stream);
     if (e != cudaSuccess) return fail(ST_ECUDA, "st7 launch (d=%d): %s", d, cudaGetErrorString(e));

@@ -43,6 +43,9 @@
 #ifndef ST7_PROF
 #define ST7_PROF 0
 #endif
+#ifndef ST7_STEADY_LOOP
+#define ST7_STEADY_LOOP (sizeof(T) == 8)   // measured: +3% FP64; FP32 D=4 spills with it
+#endif
 
 namespace st35d {
 
@@ -63,7 +66,7 @@ struct St7Params {
     int dbg;           // tuning only: bit 0 = stream planes without computing levels
     double alpha, beta;
     int split[ST7_MAX_GRID + 1];   // CTA b owns work items [split[b], split[b+1]) (host cost model)
-    unsigned long long* prof;      // ST7_PROF builds only: per-warp phase clocks [cta][warp][8]
+    unsigned long long* prof;      // ST7_PROF builds only: per-warp phase clocks [cta][warp][10]
 };
 
 constexpr int ST7_RING_MAX = 12;
@@ -333,7 +336,7 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
     // register planes: level l (1..D-1), rotating slot (prev / cur / new); level 0
     // is read straight from the TMA ring (index 0 unused)
     unsigned long long pr_t0 = ST7_PROF ? clock64() : 0, pr_wait = 0, pr_comp = 0, pr_bar = 0, pr_nr = 0, pr_ns = 0,
-                       pr_ta = 0;
+                       pr_ta = 0, pr_top = 0, pr_issue = 0, pr_gap = 0, pr_bend = 0;
     B pl[D][3];
     B outv;
 #pragma unroll
@@ -443,6 +446,7 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
             // ptxas from interleaving levels, which costs registers and moves)
             const bool ysl = yslow;
             constexpr int PREV = PH % 3, CUR = (PH + 1) % 3, NEW = (PH + 2) % 3;
+            if (ST7_PROF) { pr_top = clock64(); if (pr_bend) pr_gap += pr_top - pr_bend; }
             // issue the load of plane r + PF (its slot was freed by the barrier that ended round r-1)
             if (tid == 0) {
                 if (r + PF <= rl1) {
@@ -459,7 +463,7 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                 }
             }
             // level 0: plane r has landed in the ring
-            if (ST7_PROF) pr_ta = clock64();
+            if (ST7_PROF) { pr_ta = clock64(); pr_issue += pr_ta - pr_top; }
             if (STEADY || r <= rl1) mbar_wait(&bars[slot_r], par_r);
             unsigned long long pr_tb = 0;
             if (ST7_PROF) { pr_tb = clock64(); pr_wait += pr_tb - pr_ta; ++pr_nr; pr_ns += STEADY; }
@@ -606,7 +610,7 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
             unsigned long long pr_tc = 0;
             if (ST7_PROF) { pr_tc = clock64(); pr_comp += pr_tc - pr_tb; }
             __syncthreads();
-            if (ST7_PROF) pr_bar += clock64() - pr_tc;
+            if (ST7_PROF) { pr_bend = clock64(); pr_bar += pr_bend - pr_tc; }
             pout += plane;
             // advance the ring cursors
             slot_m2 = slot_m1;
@@ -614,25 +618,52 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
             if (++slot_r == (uint32_t)RING) { slot_r = 0; par_r ^= 1; }
             if (++slot_f == (uint32_t)RING) slot_f = 0;
         };
+        using I0 = std::integral_constant<int, 0>;
+        using I1 = std::integral_constant<int, 1>;
+        using I2 = std::integral_constant<int, 2>;
+        if (ST7_PROF) { const unsigned long long t = clock64(); pr_seg += t - pr_ts; if (!pr_first) pr_first = t - pr_t0; }
+        if constexpr (ST7_STEADY_LOOP) {
+        // Rounds of the steady range run as back-to-back phase triples with one
+        // loop branch per three rounds; the other rounds (prolog, epilog, a
+        // z-shell plane, and the few steady rounds before the phase wraps to 0)
+        // take the checked path.  ph = (r - r0) mod 3 selects the register slots.
+        int r = r0, ph = 0;
+        while (r <= r1) {
+            if (ph == 0 && r >= rs0 && r + 2 <= rs1) {
+                do {
+                    round(I0{}, std::true_type{}, r);
+                    round(I1{}, std::true_type{}, r + 1);
+                    round(I2{}, std::true_type{}, r + 2);
+                    r += 3;
+                } while (r + 2 <= rs1);
+                continue;
+            }
+            const bool st = r >= rs0 && r <= rs1;
+            if (ph == 0) { if (st) round(I0{}, std::true_type{}, r); else round(I0{}, std::false_type{}, r); }
+            else if (ph == 1) { if (st) round(I1{}, std::true_type{}, r); else round(I1{}, std::false_type{}, r); }
+            else { if (st) round(I2{}, std::true_type{}, r); else round(I2{}, std::false_type{}, r); }
+            ++r;
+            ph = ph == 2 ? 0 : ph + 1;
+        }
+        } else {
         auto any_round = [&](auto PHc, int r) {
             if (r >= rs0 && r <= rs1) round(PHc, std::true_type{}, r);
             else round(PHc, std::false_type{}, r);
         };
-
-        if (ST7_PROF) { const unsigned long long t = clock64(); pr_seg += t - pr_ts; if (!pr_first) pr_first = t - pr_t0; }
         for (int r = r0; r <= r1;) {
-            any_round(std::integral_constant<int, 0>{}, r);
+            any_round(I0{}, r);
             if (++r > r1) break;
-            any_round(std::integral_constant<int, 1>{}, r);
+            any_round(I1{}, r);
             if (++r > r1) break;
-            any_round(std::integral_constant<int, 2>{}, r);
+            any_round(I2{}, r);
             ++r;
+        }
         }
     }
     if (ST7_PROF && p.prof && (tid & 31) == 0) {
-        unsigned long long* o = p.prof + ((size_t)blockIdx.x * (MAXT / 32) + tid / 32) * 8;
+        unsigned long long* o = p.prof + ((size_t)blockIdx.x * (MAXT / 32) + tid / 32) * 10;
         o[0] = clock64() - pr_t0; o[1] = pr_wait; o[2] = pr_comp; o[3] = pr_bar; o[4] = pr_nr; o[5] = pr_ns;
-        o[6] = pr_seg; o[7] = pr_first;
+        o[6] = pr_seg; o[7] = pr_first; o[8] = pr_issue; o[9] = pr_gap;
     }
 }
 

@@ -15,9 +15,9 @@ os.remove(out)
 p.st7(x, y, 0.4, 0.1, D); p.sync()      # one sweep, profiled
 b = open(out, 'rb').read()
 grid, wpc, d, nzo = struct.unpack('4i', b[:16])
-a = np.frombuffer(b[16:], dtype=np.uint64)[:grid * wpc * 8].reshape(grid, wpc, 8).astype(np.float64)
+a = np.frombuffer(b[16:], dtype=np.uint64)[:grid * wpc * 10].reshape(grid, wpc, 10).astype(np.float64)
 a = a[:, :max(1, wpc - (1 if a[0, -1, 4] == 0 else 0))]
-tot, wait, comp, bar, nr, ns, seg, first = (a[..., i] for i in range(8))
+tot, wait, comp, bar, nr, ns, seg, first, issue, gap = (a[..., i] for i in range(10))
 act = nr[..., ] > 0
 print(f"N={n} D={d} {dt} grid={grid} warps/cta={wpc}")
 print(f"  kernel clocks per CTA: mean {tot[:,0].mean():.0f} max {tot[:,0].max():.0f} min {tot[:,0].min():.0f}")
@@ -26,6 +26,7 @@ r = nr[:, :].clip(1)
 print(f"  per round (mean over warps): wait {(wait/r).mean():.0f}  compute {(comp/r).mean():.0f}  barrier {(bar/r).mean():.0f}  total {(tot/r).mean():.0f}")
 print(f"  compute per round by warp (CTA 0): {np.round(comp[0]/r[0]).astype(int).tolist()}")
 print(f"  barrier per round by warp (CTA 0): {np.round(bar[0]/r[0]).astype(int).tolist()}")
+print(f"  per round: TMA-issue block {(issue/r).mean():.0f} (warp 0: {(issue[:,0]/r[:,0]).mean():.0f}), barrier-end -> next round {(gap/r).mean():.0f}")
 print(f"  outside rounds (setup, segment switch) per CTA: {(tot - wait - comp - bar)[:,0].mean():.0f}")
 print(f"  segment setup per CTA: {seg[:,0].mean():.0f} (first round starts at {first[:,0].mean():.0f})")
 print(f"  rounds per CTA histogram: {np.bincount(nr[:,0].astype(int)).nonzero()[0].tolist()}")
