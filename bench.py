@@ -365,6 +365,9 @@ def main():
             pn.set_stream(stream)
             pn.set_variant(st.ST_VARIANT_NAIVE)
             tn, _ = time_steps(lambda: pn.st7(xa, ya, 0.4, 0.1, T), 2, 1)
+        with st.Plan(n, n, n, torch.float32, 8) as pa:   # the library's own depth selection (f3)
+            pa.set_stream(stream)
+            at_d, at_eta, at_ms = pa.autotune(xa, ya, 24)
         del xa, ya
         gamma = 8.0 / ST7_OPS                                    # B per FP instruction
         Gamma = hbm_gbs * 1e9 / (ops_peak * 1e12)                # B200: measured HBM / FP32 lane-instr rate
@@ -374,6 +377,8 @@ def main():
             "2.5D_dim_T_1": sweep.get(1), "3.5D": round(value, 1), "dim_T": D,
             "model": {"gamma_B_per_instr": round(gamma, 3), "Gamma_B_per_instr": round(Gamma, 4),
                       "eta_eq3": mdl["eta"], "measured_best_dim_T": D,
+                      "st_plan_autotune": {"dim_T": at_d, "eta_seed_nominal_peaks": at_eta, "T_probe": 24,
+                                           "ms": {k: round(v, 4) for k, v in at_ms.items()}},
                       "note": "eta = ceil(gamma/Gamma) is where the HBM roof meets the FP32 roof; the "
                               "measured optimum is lower because the kernel is issue/latency-bound"}}
         # LBM D3Q19 cavity 256^3 (configs[2])

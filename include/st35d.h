@@ -132,6 +132,20 @@ int st_plan_set_bitexact(st_plan* plan, int on);
 enum { ST_VARIANT_35D = 0, ST_VARIANT_NAIVE = 1 };
 int st_plan_set_variant(st_plan* plan, int variant);
 
+/* st_plan_autotune — choose the 7-point sweep depth by measurement (the
+ * paper's "framework that determines the various blocking parameters", P:377,
+ * eqs. (1)-(4) of §V-C).  Every depth 1..(deepest the plan tiles, <= dim_T)
+ * runs T_probe Jacobi steps of st7_run on the caller's DEVICE grids a and b
+ * (n^3 each, both clobbered), timed with CUDA events on the plan stream; the
+ * fastest depth becomes the plan's st7_run sweep depth (results are identical
+ * for every depth).  eta_out (may be NULL) receives the eq. (3) seed
+ * eta = ceil(gamma/Gamma) with gamma = 2E/7 bytes per FP instruction and Gamma
+ * = this device's nominal HBM bytes/s over its FP32 (FP64) lane-instr/s;
+ * ms_out (may be NULL, length >= dim_T) receives the time per depth.
+ * Synchronous.  Single-process plans only (ST_EUNSUPPORTED otherwise: tune
+ * one rank and broadcast).  Returns the chosen depth (>= 1) or < 0. */
+int st_plan_autotune(st_plan* plan, void* a, void* b, int T_probe, int* eta_out, float* ms_out);
+
 /* Waits for the plan stream; returns ST_ECUDA for deferred device faults. */
 int st_plan_sync(st_plan* plan);
 

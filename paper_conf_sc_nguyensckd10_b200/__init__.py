@@ -46,7 +46,7 @@ class st_blocking(ctypes.Structure):
 _lib = None
 
 EXPORTS = ["st_plan_create", "st7_run", "lbm_d3q19_run", "st_destroy", "st_last_error", "st_last_status",
-           "st_plan_set_stream", "st_plan_set_lbm_lid", "st_plan_set_bitexact", "st_plan_set_variant", "st_plan_sync",
+           "st_plan_set_stream", "st_plan_set_lbm_lid", "st_plan_set_bitexact", "st_plan_set_variant", "st_plan_autotune", "st_plan_sync",
            "st_plan_set_dist", "st_plan_set_loopback_slabs", "st_plan_ghost_planes", "st_plan_local_slab",
            "st_plan_get_info", "st_plan_last_launches", "st_blocking_model", "st_fig3_step",
            "st_nccl_unique_id", "st_slab_range"]
@@ -72,6 +72,7 @@ def lib() -> ctypes.CDLL:
         "st_plan_set_lbm_lid": ([P, D, D, D], I),
         "st_plan_set_bitexact": ([P, I], I),
         "st_plan_set_variant": ([P, I], I),
+        "st_plan_autotune": ([P, P, P, I, ctypes.POINTER(I), ctypes.POINTER(ctypes.c_float)], I),
         "st_plan_sync": ([P], I),
         "st_plan_set_dist": ([P, P, I, I], I),
         "st_plan_set_loopback_slabs": ([P, I], I),
@@ -160,6 +161,14 @@ def st_plan_set_variant(plan: int, variant: int) -> int:
     return _check(lib().st_plan_set_variant(plan, int(variant)))
 
 
+def st_plan_autotune(plan: int, a, b, T_probe: int):
+    """returns (chosen dim_T, eq. (3) eta seed, {dim_T: ms for T_probe steps})."""
+    eta = ctypes.c_int()
+    ms = (ctypes.c_float * 16)()
+    d = _check(lib().st_plan_autotune(plan, _ptr(a), _ptr(b), T_probe, ctypes.byref(eta), ms))
+    return d, eta.value, {k + 1: ms[k] for k in range(16) if ms[k] > 0}
+
+
 def st_plan_sync(plan: int) -> int:
     return _check(lib().st_plan_sync(plan))
 
@@ -242,6 +251,9 @@ class Plan:
 
     def set_stream(self, stream) -> None:
         st_plan_set_stream(self.h, stream)
+
+    def autotune(self, a, b, T_probe: int):
+        return st_plan_autotune(self.h, a, b, T_probe)
 
     def set_variant(self, variant: int) -> None:
         st_plan_set_variant(self.h, variant)

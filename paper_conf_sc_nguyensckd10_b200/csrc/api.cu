@@ -91,7 +91,8 @@ struct st_plan {
     int nx, ny, nz;
     st_dtype dtype;
     int dimT;
-    int dimK = 0;      // deepest sweep the 7-point kernels can tile (<= dimT)
+    int dimK = 0;      // sweep depth of st7_run (<= dimT; st_plan_autotune may lower it)
+    int dimKmax = 0;   // deepest sweep the 7-point kernels can tile (<= dimT)
     int dev = 0, sms = 0;
     size_t smem_optin = 0;
     cudaStream_t stream = nullptr;
@@ -252,7 +253,7 @@ extern "C" st_plan* st_plan_create(int nx, int ny, int nz, st_dtype dtype, int d
     // those plans run sweeps of depth dimK < dim_T; results are identical)
     Geo7* g = nullptr;
     for (int d = dim_T; d >= 1; --d)
-        if (get_geo7(p, d, nz, g) == ST_OK) { p->dimK = d; break; }
+        if (get_geo7(p, d, nz, g) == ST_OK) { p->dimK = p->dimKmax = d; break; }
     if (!p->dimK) { st_destroy(p); return nullptr; }
     g_err.clear();
     g_code = 0;
@@ -731,6 +732,62 @@ extern "C" int st7_run(st_plan* p, const void* in, void* out, double alpha, doub
     CUDA_TRY(cudaMemcpyAsync(out, p->hbuf[1], n, cudaMemcpyDeviceToHost, p->stream));
     CUDA_TRY(cudaStreamSynchronize(p->stream));
     return ST_OK;
+}
+
+// ----------------------------------------------------------------------------
+// Blocking-parameter selection by measurement ("a framework that
+// determines the various blocking parameters"): the eq. (3) bound eta from this
+// device's HBM bandwidth and FP issue rate seeds the report; every depth
+// 1..dimKmax is timed on the caller's grids and the fastest is kept.
+// ----------------------------------------------------------------------------
+extern "C" int st_plan_autotune(st_plan* p, void* a, void* b, int T_probe, int* eta_out, float* ms_out) {
+    if (!p) return fail(ST_EINVAL, "NULL plan");
+    if (!a || !b) return fail(ST_EINVAL, "NULL grid pointer");
+    if (T_probe < 1) return fail(ST_EINVAL, "T_probe = %d < 1", T_probe);
+    if (p->dist.mode != Dist::SINGLE) return fail(ST_EUNSUPPORTED, "autotune a single-process plan and broadcast");
+    const size_t n = (size_t)p->nx * p->ny * p->dist.nzb * esize(p->dtype);
+    if (overlap(a, b, n)) return fail(ST_EINVAL, "a and b overlap");
+    if (ptr_kind(a) != 1 || ptr_kind(b) != 1) return fail(ST_EINVAL, "autotune needs device grids");
+    if ((reinterpret_cast<uintptr_t>(a) | reinterpret_cast<uintptr_t>(b)) & 15)
+        return fail(ST_EINVAL, "device grids must be 16-byte aligned");
+    if (eta_out) {   // eq. (3): gamma = 2E bytes / 7 FP instructions per update; Gamma of this device
+        int memclk_khz = 0, bus_bits = 0, smclk_khz = 0;
+        cudaDeviceGetAttribute(&memclk_khz, cudaDevAttrMemoryClockRate, p->dev);
+        cudaDeviceGetAttribute(&bus_bits, cudaDevAttrGlobalMemoryBusWidth, p->dev);
+        cudaDeviceGetAttribute(&smclk_khz, cudaDevAttrClockRate, p->dev);
+        const double lanes = p->dtype == ST_F32 ? 128.0 : 64.0;   // FP32 / FP64 lanes per SM (sm_100)
+        const double bw = 2.0 * memclk_khz * 1e3 * bus_bits / 8.0;
+        const double ops = (double)p->sms * lanes * smclk_khz * 1e3;
+        st_blocking m{};
+        const double E = (double)esize(p->dtype);
+        *eta_out = (bw > 0 && ops > 0 && st_blocking_model(p->smem_optin, E, 1, 2.0 * E / 7.0, bw / ops, 0, 0, &m) == ST_OK)
+                       ? m.eta : 0;
+    }
+    cudaEvent_t e0, e1;
+    CUDA_TRY(cudaEventCreate(&e0));
+    CUDA_TRY(cudaEventCreate(&e1));
+    const int keep = p->dimK;
+    int best = keep;
+    float best_ms = 0.f;
+    int rc = ST_OK;
+    for (int d = 1; d <= p->dimKmax && rc == ST_OK; ++d) {
+        p->dimK = d;
+        rc = run7_device(p, a, b, 0.4, 0.1, std::min(T_probe, 2 * d));   // warm-up (geometry, first launch)
+        if (rc) break;
+        cudaEventRecord(e0, p->stream);
+        rc = run7_device(p, a, b, 0.4, 0.1, T_probe);
+        if (rc) break;
+        cudaEventRecord(e1, p->stream);
+        if (cudaEventSynchronize(e1) != cudaSuccess) { rc = fail(ST_ECUDA, "autotune: %s", cudaGetErrorString(cudaGetLastError())); break; }
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, e0, e1);
+        if (ms_out) ms_out[d - 1] = ms;
+        if (d == 1 || ms < best_ms) { best = d; best_ms = ms; }
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    p->dimK = rc ? keep : best;
+    return rc ? rc : best;
 }
 
 // ----------------------------------------------------------------------------

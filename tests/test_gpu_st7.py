@@ -150,3 +150,25 @@ def test_naive_variant_bitexact(oracle_lib, dtype, T):
         p.sync()
         assert p.last_launches() == T
     assert np.array_equal(y.cpu().numpy(), ref)
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_autotune_picks_a_depth_and_stays_exact(oracle_lib, dtype):
+    # st_plan_autotune times every depth and keeps the fastest; results are depth-independent
+    nx, ny, nz = 96, 72, 40
+    dt = torch.float32 if dtype == np.float32 else torch.float64
+    a = stgen.grid7(nx, ny, nz, 11, dtype)
+    ref = oracle_lib.st7(a, 0.4, 0.1, 9)
+    with st.Plan(nx, ny, nz, dt, 6) as p:
+        x = torch.empty(nz, ny, nx, dtype=dt, device="cuda")
+        y = torch.empty_like(x)
+        d, eta, ms = p.autotune(x, y, 6)
+        assert 1 <= d <= 6 and eta >= 1
+        assert sorted(ms) == list(range(1, len(ms) + 1)) and d in ms
+        assert ms[d] == min(ms.values())
+        assert p.info()["dim_t_sweep"] == d
+        p.set_bitexact(True)
+        x.copy_(torch.from_numpy(a))
+        p.st7(x, y, 0.4, 0.1, 9)
+        p.sync()
+    assert np.array_equal(y.cpu().numpy(), ref)
