@@ -333,9 +333,10 @@ extern "C" int st_plan_get_info(const st_plan* p, int lbm, st_plan_info* info) {
         info->dim_t_sweep = d;
         return ST_OK;
     }
-    auto it = p->geo7.find(p->dimK);
-    if (it == p->geo7.end()) return fail(ST_EINVAL, "no plan for dim_T");
-    const Geo7& g = it->second;
+    Geo7* gp = nullptr;   // geometry of the plan's sweep depth (built on demand)
+    int rc = get_geo7(const_cast<st_plan*>(p), p->dimK, p->dist.nzl, gp);
+    if (rc) return rc;
+    const Geo7& g = *gp;
     info->tile_x = g.TX; info->tile_y = g.TY; info->out_x = g.wx; info->out_y = g.wy;
     info->tiles_x = g.tiles_x; info->tiles_y = g.tiles_y; info->ctas = g.grid; info->threads = g.threads;
     info->smem_bytes = (int)g.smem; info->kappa = g.kappa; info->kernel = g.VY * 1000 + g.maxt + (g.split ? 100000 : 0);
