@@ -403,6 +403,38 @@ def main():
                                                          "frac": round(gbs / hbm_gbs, 4)},
                                             "launches": pl.last_launches()}
             del fa, fb, f0, flags
+        # configs[4] lattice on one GPU (1024^3 FP32 cavity from rest: the strong-scaling base,
+        # 163 GB for the two lattices), built on the device
+        torch.cuda.empty_cache()
+        nb = 1024
+        if torch.cuda.mem_get_info()[0] >= 2 * 19 * nb ** 3 * 4 + 3 * nb ** 3 + (4 << 30):
+            flb = torch.zeros((nb, nb, nb), dtype=torch.uint8, device="cuda")
+            flb[:, 0, :] = 1
+            flb[:, :, 0] = 1
+            flb[:, :, nb - 1] = 1
+            flb[0] = 1
+            flb[nb - 1] = 1
+            flb[:, nb - 1, :] = 2
+            fa = torch.empty((19, nb, nb, nb), dtype=torch.float32, device="cuda")
+            wv = stgen.lbm_rest(1, 1, 1, np.float32).reshape(19)
+            for i in range(19):
+                fa[i].fill_(float(wv[i]))
+            fb = torch.empty_like(fa)
+            Tb = 10
+            with st.Plan(nb, nb, nb, torch.float32, 1) as pl:
+                pl.set_stream(stream)
+                pl.set_lid(0.05, 0.0, 0.0)
+                tl, _ = time_steps(lambda: pl.lbm(fa, fb, 1.6, Tb, flb), 2, 1)
+                msl = tl / 2
+                cells = (nb - 2) ** 3
+                gbs = LBM_BYTES[4] * cells * Tb / (msl / 1e3) / 1e9
+                extras["lbm_f32_1024"] = {"value": round(cells * Tb / (msl / 1e3) / 1e6, 1), "unit": "MLUPS",
+                                          "dim_T": 1, "T": Tb, "ms_per_step": round(msl, 3),
+                                          "note": "configs[4] lattice on one GPU (strong-scaling base)",
+                                          "roofline": {"bound": "hbm", "achieved": round(gbs, 1), "peak": hbm_gbs,
+                                                       "unit": "GB/s", "frac": round(gbs / hbm_gbs, 4)}}
+            del fa, fb, flb
+            torch.cuda.empty_cache()
     cpu = cpu_baseline_7pt(n) if (rank == 0 and world == 1) else None
 
     if rank == 0:

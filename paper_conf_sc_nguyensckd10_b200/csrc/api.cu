@@ -872,8 +872,8 @@ static int launch_lbm(st_plan* p, const void* src, void* dst, const uint8_t* fla
     else lid_coeffs<double>(p->lid, prm.lidc);
     const long long cells = (long long)(sv.zb - sv.za) * p->nx * p->ny;
     if (cells <= 0) return ST_OK;
-    // one wave of resident 256-thread CTAs (launch bounds: 4 per SM FP32, 2 FP64), grid-stride over the cells
-    int bps = p->dtype == ST_F32 ? 4 : 2;
+    // one wave of resident 256-thread CTAs (launch bounds: 4 per SM, 2 for the batched-flag kernel), grid-stride
+    int bps = lbm_push_batched((int)esize(p->dtype), p->nx, p->ny, sv.nzb) ? 2 : 4;
     if (const char* e = getenv("ST_LBM_BPS")) bps = std::max(1, atoi(e));   // A/B tuning
     const int grid = (int)std::min<long long>((cells + 255) / 256, (long long)p->sms * bps);
     cudaError_t e = lbm_push_launch(p->dtype == ST_F32 ? 0 : 1, p->exact, src, dst, sv.fl2, prm, grid,

@@ -1,7 +1,19 @@
 // lbm_inst.cu — instantiates the LBM kernels and the shell-flag check.
+#include <cstdlib>
 #include "launch.h"
 
 namespace st35d {
+
+// FP32 lattices of more than 2^24 cells run the batched-flag kernel at 2
+// CTAs/SM: it holds 23-27 GLUPS from 320^3 to 1024^3 (22.7 vs 15.4 at 1024^3,
+// 22.9 vs 18.5 at 512^3, 26.6 vs 20.2 at 448^3), while the per-direction
+// kernel at 4 CTAs/SM swings with the lattice size and is 3 % faster only up to
+// 256^3 (tools/lbm_big.py, T = 20); FP64 always batches.  ST_LBM_BATCH=0/1
+// overrides (A/B).
+bool lbm_push_batched(int esize, int nx, int ny, int nzb) {
+    if (const char* e = getenv("ST_LBM_BATCH")) return atoi(e) != 0;
+    return esize == 8 || (long long)nx * ny * nzb > (1LL << 24);
+}
 
 template <typename T, bool E>
 static cudaError_t push_t(const void* src, void* dst, const uint8_t* fl2, const LbmParams& p, int grid,
@@ -9,10 +21,16 @@ static cudaError_t push_t(const void* src, void* dst, const uint8_t* fl2, const 
     // FP64: 32-bit element offsets when every population offset (and a plane step)
     // fits; FP32 keeps 64-bit offsets (measured 26.0 vs 23.6 GLUPS at 256^3, tools/lbm_ab.sh)
     const long long span = 20LL * p.nx * p.ny * p.nzb;
-    if (sizeof(T) == 8 && span < (1LL << 31))
-        lbm_push_kernel<T, E, int><<<grid, 256, 0, s>>>(static_cast<const T*>(src), static_cast<T*>(dst), fl2, p);
-    else
-        lbm_push_kernel<T, E, long long><<<grid, 256, 0, s>>>(static_cast<const T*>(src), static_cast<T*>(dst), fl2, p);
+    const T* a = static_cast<const T*>(src);
+    T* b = static_cast<T*>(dst);
+    if (sizeof(T) == 8) {
+        if (span < (1LL << 31)) lbm_push_kernel<T, E, int, true><<<grid, 256, 0, s>>>(a, b, fl2, p);
+        else lbm_push_kernel<T, E, long long, true><<<grid, 256, 0, s>>>(a, b, fl2, p);
+    } else if (lbm_push_batched(4, p.nx, p.ny, p.nzb)) {
+        lbm_push_kernel<T, E, long long, true><<<grid, 256, 0, s>>>(a, b, fl2, p);
+    } else {
+        lbm_push_kernel<T, E, long long, false><<<grid, 256, 0, s>>>(a, b, fl2, p);
+    }
     return cudaGetLastError();
 }
 

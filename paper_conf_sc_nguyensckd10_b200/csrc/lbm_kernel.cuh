@@ -144,11 +144,10 @@ __device__ __forceinline__ void collide(T (&f)[19], T omega) {
 // of bursting them into the LSU queue ahead of other warps' loads — while
 // FP64 (twice the bytes per store) prefers all 18 neighbour flags loaded up
 // front (one round trip), 17.0 vs 15.7 GLUPS.
-template <typename T, bool E, typename IX>
-__global__ void __launch_bounds__(256, (sizeof(T) == 4 ? 4 : 2))
+template <typename T, bool E, typename IX, bool BATCH>
+__global__ void __launch_bounds__(256, (BATCH ? 2 : 4))
 lbm_push_kernel(const T* __restrict__ src, T* __restrict__ dst, const uint8_t* __restrict__ fl2,
                 const LbmParams p) {
-    constexpr bool BATCH = sizeof(T) == 8;
     const size_t plane = (size_t)p.nx * p.ny;
     const size_t nc = plane * p.nzb;              // SoA stride of one population
     const size_t c0 = (size_t)p.za * plane;

@@ -127,3 +127,63 @@ def test_flags_rewritten_in_place(oracle_lib):
         p.lbm(a, b, 1.3, 4, fl)
         p.sync()
         assert np.array_equal(b.cpu().numpy(), oracle_lib.lbm(f0, flags2, 1.3, 4))
+
+
+def _cavity_on_device(n, dtype):
+    """configs[4]-size cavity from rest built on the device (a 1024^3 lattice does not fit host-side)."""
+    fl = torch.zeros((n, n, n), dtype=torch.uint8, device="cuda")
+    fl[:, 0, :] = stgen.WALL
+    fl[:, :, 0] = stgen.WALL
+    fl[:, :, n - 1] = stgen.WALL
+    fl[0] = stgen.WALL
+    fl[n - 1] = stgen.WALL
+    fl[:, n - 1, :] = stgen.LID
+    f = torch.empty((19, n, n, n), dtype=dtype, device="cuda")
+    w = stgen.lbm_rest(1, 1, 1, np.float32 if dtype == torch.float32 else np.float64).reshape(19)
+    for i in range(19):
+        f[i].fill_(float(w[i]))
+    return f, fl
+
+
+def test_config4_lbm_1024_light_cone(oracle_lib):
+    # configs[4] lattice (1024^3 FP32 cavity, the strong-scaling base) on one GPU, bit-exact
+    # build.  After T steps from rest a cell depends only on its radius-T neighbourhood
+    # (one lattice link per step), so windows at the lid centre, at lid corners, at a
+    # bottom corner and at the centre must equal the same windows of the oracle run on a
+    # small cavity with the same local geometry; every shifted window has its light cone
+    # inside both lattices.  Fluid mass is conserved (P8b) over the whole lattice.
+    n, T = 1024, 3
+    need = 2 * 19 * n ** 3 * 4 + 3 * n ** 3 + (4 << 30)
+    if torch.cuda.mem_get_info()[0] < need:
+        pytest.skip("1024^3 FP32 lattice pair does not fit this device")
+    f, fl = _cavity_on_device(n, torch.float32)
+    g = torch.empty_like(f)
+    w = stgen.lbm_rest(1, 1, 1, np.float32).reshape(19).astype(np.float64)
+    mass0 = float(w.sum()) * (n - 2) ** 3
+    with st.Plan(n, n, n, torch.float32, 1) as p:
+        p.set_lid(0.05, 0.0, 0.0)
+        p.set_bitexact(True)
+        p.lbm(f, g, 1.6, T, fl)
+        p.sync()
+    del f
+    ns = 2 * T + 8
+    ref = oracle_lib.lbm(stgen.lbm_rest(ns, ns, ns, np.float32), stgen.cavity_flags(ns, ns, ns), 1.6, T)
+    h, c, cs = T + 3, n // 2, ns // 2
+    windows = [   # (big z, y, x slices), (small z, y, x slices)
+        ((slice(c - 2, c + 3), slice(n - h, n), slice(c - 2, c + 3)),
+         (slice(cs - 2, cs + 3), slice(ns - h, ns), slice(cs - 2, cs + 3))),        # lid centre
+        ((slice(0, h), slice(n - h, n), slice(0, h)), (slice(0, h), slice(ns - h, ns), slice(0, h))),   # lid corner
+        ((slice(n - h, n), slice(n - h, n), slice(n - h, n)),
+         (slice(ns - h, ns), slice(ns - h, ns), slice(ns - h, ns))),                 # far lid corner
+        ((slice(0, h), slice(0, h), slice(0, h)), (slice(0, h), slice(0, h), slice(0, h))),   # bottom corner
+        ((slice(c - 1, c + 2), slice(c - 1, c + 2), slice(c - 1, c + 2)),
+         (slice(cs - 1, cs + 2), slice(cs - 1, cs + 2), slice(cs - 1, cs + 2))),     # centre
+    ]
+    for big, small in windows:
+        got = g[(slice(None),) + big].cpu().numpy()
+        assert np.array_equal(got, ref[(slice(None),) + small])
+    mass = 0.0
+    for i in range(19):
+        for z0 in range(1, n - 1, 64):
+            mass += float(g[i, z0:min(z0 + 64, n - 1), 1:n - 1, 1:n - 1].double().sum())
+    assert abs(mass - mass0) <= 1e-6 * mass0
