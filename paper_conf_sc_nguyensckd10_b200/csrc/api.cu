@@ -870,13 +870,15 @@ static int launch_lbm(st_plan* p, const void* src, void* dst, const uint8_t* fla
     prm.omega = omega;
     if (p->dtype == ST_F32) lid_coeffs<float>(p->lid, prm.lidc);
     else lid_coeffs<double>(p->lid, prm.lidc);
-    const long long cells = (long long)(sv.zb - sv.za) * p->nx * p->ny;
-    if (cells <= 0) return ST_OK;
+    // Z-slab views also process the ghost planes next to the output planes (push form)
+    const int pa = sv.single ? sv.za : std::max(sv.za - 1, 0), pb = sv.single ? sv.zb : std::min(sv.zb + 1, sv.nzb);
+    const long long cells = (long long)(pb - pa) * p->nx * p->ny;
+    if (cells <= 0 || sv.zb <= sv.za) return ST_OK;
     // one wave of resident 256-thread CTAs (launch bounds: 4 per SM, 2 for the batched-flag kernel), grid-stride
     int bps = lbm_push_batched((int)esize(p->dtype), p->nx, p->ny, sv.nzb) ? 2 : 4;
     if (const char* e = getenv("ST_LBM_BPS")) bps = std::max(1, atoi(e));   // A/B tuning
     const int grid = (int)std::min<long long>((cells + 255) / 256, (long long)p->sms * bps);
-    cudaError_t e = lbm_push_launch(p->dtype == ST_F32 ? 0 : 1, p->exact, src, dst, sv.fl2, prm, grid,
+    cudaError_t e = lbm_push_launch(p->dtype == ST_F32 ? 0 : 1, p->exact, !sv.single, src, dst, sv.fl2, prm, grid,
                                     sv.stream ? sv.stream : p->stream);
     if (e != cudaSuccess) return fail(ST_ECUDA, "lbm launch: %s", cudaGetErrorString(e));
     ++p->launches;
@@ -907,7 +909,7 @@ static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T
     }
     // dim_T = 1: the fused push kernel (fastest measured on B200); dim_T >= 2:
     // the on-chip multi-level sweep lbm_35d (ST_LBM_35D=1 forces it for dim_T = 1)
-    const bool push = max_lbm_depth(p) == 1 && getenv("ST_LBM_35D") == nullptr && p->dist.mode == Dist::SINGLE;
+    const bool push = max_lbm_depth(p) == 1 && getenv("ST_LBM_35D") == nullptr;
     // neighbour-flag prepass, every call (a reused flags pointer may hold new contents; ~1 pass over the flags)
     if (p->dist.mode != Dist::LOOPBACK) {
         const size_t cells = (size_t)p->nx * p->ny * p->dist.nzb;

@@ -43,7 +43,7 @@ St7LaunchFn st7s_lookup_f64_fast(int D, int VY, int MAXT);
 St7LaunchFn st7s_lookup_f64_exact(int D, int VY, int MAXT);
 
 bool lbm_push_batched(int esize, int nx, int ny, int nzb);   // kernel choice (also sets the grid)
-cudaError_t lbm_push_launch(int dtype, bool exact, const void* src, void* dst, const uint8_t* fl2,
+cudaError_t lbm_push_launch(int dtype, bool exact, bool slab, const void* src, void* dst, const uint8_t* fl2,
                             const LbmParams& p, int grid, cudaStream_t s);
 cudaError_t lbm35_launch(int dtype, bool exact, int D, const Lbm35Params& p, int grid, int threads, size_t smem,
                          cudaStream_t s);

@@ -15,7 +15,7 @@ bool lbm_push_batched(int esize, int nx, int ny, int nzb) {
     return esize == 8 || (long long)nx * ny * nzb > (1LL << 24);
 }
 
-template <typename T, bool E>
+template <typename T, bool E, bool SLAB>
 static cudaError_t push_t(const void* src, void* dst, const uint8_t* fl2, const LbmParams& p, int grid,
                           cudaStream_t s) {
     // FP64: 32-bit element offsets when every population offset (and a plane step)
@@ -24,22 +24,29 @@ static cudaError_t push_t(const void* src, void* dst, const uint8_t* fl2, const 
     const T* a = static_cast<const T*>(src);
     T* b = static_cast<T*>(dst);
     if (sizeof(T) == 8) {
-        if (span < (1LL << 31)) lbm_push_kernel<T, E, int, true><<<grid, 256, 0, s>>>(a, b, fl2, p);
-        else lbm_push_kernel<T, E, long long, true><<<grid, 256, 0, s>>>(a, b, fl2, p);
+        if (span < (1LL << 31)) lbm_push_kernel<T, E, int, true, SLAB><<<grid, 256, 0, s>>>(a, b, fl2, p);
+        else lbm_push_kernel<T, E, long long, true, SLAB><<<grid, 256, 0, s>>>(a, b, fl2, p);
     } else if (lbm_push_batched(4, p.nx, p.ny, p.nzb)) {
-        lbm_push_kernel<T, E, long long, true><<<grid, 256, 0, s>>>(a, b, fl2, p);
+        lbm_push_kernel<T, E, long long, true, SLAB><<<grid, 256, 0, s>>>(a, b, fl2, p);
     } else {
-        lbm_push_kernel<T, E, long long, false><<<grid, 256, 0, s>>>(a, b, fl2, p);
+        lbm_push_kernel<T, E, long long, false, SLAB><<<grid, 256, 0, s>>>(a, b, fl2, p);
     }
     return cudaGetLastError();
 }
 
+template <typename T, bool E>
+static cudaError_t push_s(bool slab, const void* src, void* dst, const uint8_t* fl2, const LbmParams& p, int grid,
+                          cudaStream_t s) {
+    return slab ? push_t<T, E, true>(src, dst, fl2, p, grid, s) : push_t<T, E, false>(src, dst, fl2, p, grid, s);
+}
+
 // fl2 = the lbm_fl2 prepass output of the flags
-cudaError_t lbm_push_launch(int dtype, bool exact, const void* src, void* dst, const uint8_t* fl2,
+cudaError_t lbm_push_launch(int dtype, bool exact, bool slab, const void* src, void* dst, const uint8_t* fl2,
                             const LbmParams& p, int grid, cudaStream_t s) {
-    if (dtype == 0) return exact ? push_t<float, true>(src, dst, fl2, p, grid, s)
-                                 : push_t<float, false>(src, dst, fl2, p, grid, s);
-    return exact ? push_t<double, true>(src, dst, fl2, p, grid, s) : push_t<double, false>(src, dst, fl2, p, grid, s);
+    if (dtype == 0) return exact ? push_s<float, true>(slab, src, dst, fl2, p, grid, s)
+                                 : push_s<float, false>(slab, src, dst, fl2, p, grid, s);
+    return exact ? push_s<double, true>(slab, src, dst, fl2, p, grid, s)
+                 : push_s<double, false>(slab, src, dst, fl2, p, grid, s);
 }
 
 template <typename T, int D, bool E>
