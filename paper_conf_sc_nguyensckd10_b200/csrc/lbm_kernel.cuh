@@ -144,77 +144,100 @@ __device__ __forceinline__ void collide(T (&f)[19], T omega) {
 // of bursting them into the LSU queue ahead of other warps' loads — while
 // FP64 (twice the bytes per store) prefers all 18 neighbour flags loaded up
 // front (one round trip), 17.0 vs 15.7 GLUPS.
+// constants of one push sweep (see lbm_push_kernel)
+template <typename IX> struct PushCtx {
+    size_t plane, lo0, lo1, hi0, hi1, last;
+    IX ncx, pl;
+    int nx;
+};
+
+// collide one cell (populations f, flag fl) and push its 19 values (or copy a
+// non-FLUID cell through).  SLAB: only stores into the output planes are kept.
+template <typename T, bool E, typename IX, bool BATCH, bool SLAB>
+__device__ __forceinline__ void lbm_push_cell(T (&f)[19], uint32_t fl, size_t c, const uint8_t* __restrict__ fl2,
+                                              T* __restrict__ dst, const PushCtx<IX>& k, T omega, const LbmParams& p) {
+    const bool own = !SLAB || (c >= k.lo0 && c < k.hi1);
+    const bool dn_ok = !SLAB || c >= k.lo1;     // target plane q-1 >= za
+    const bool up_ok = !SLAB || c < k.hi0;      // target plane q+1 < zb
+    T* __restrict__ d = dst + c;
+    if (fl & 0x7fu) {   // WALL / LID: copied through
+        if (own) {
+#pragma unroll
+            for (int i = 0; i < 19; ++i) d[(IX)i * k.ncx] = f[i];
+        }
+        return;
+    }
+    collide<T, E>(f, omega);
+    uint32_t tfl[19];
+    if constexpr (BATCH) {
+        auto ld = [&](auto Ic) {
+            constexpr int I = decltype(Ic)::value;
+            const IX off = (IX)D3Q19<I>::ex + (IX)D3Q19<I>::ey * (IX)k.nx + (IX)D3Q19<I>::ez * k.pl;
+            // (SLAB: a neighbour outside the buffer is never a store target; read nothing)
+            const bool in = !SLAB || (D3Q19<I>::ez < 0 ? c >= k.plane : (D3Q19<I>::ez > 0 ? c < k.last : true));
+            tfl[I] = (I == 0 || !in) ? 0u : (uint32_t)__ldg(fl2 + c + off);
+        };
+        [&]<int... Is>(std::integer_sequence<int, Is...>) { (ld(std::integral_constant<int, Is>{}), ...); }
+        (std::make_integer_sequence<int, 19>{});
+    }
+    auto push = [&](auto Ic) {
+        constexpr int I = decltype(Ic)::value;
+        constexpr int ez = D3Q19<I>::ez;
+        const IX off = (IX)D3Q19<I>::ex + (IX)D3Q19<I>::ey * (IX)k.nx + (IX)ez * k.pl;
+        const bool tgt_ok = ez < 0 ? dn_ok : (ez > 0 ? up_ok : own);
+        if constexpr (I == 0) {
+            if (own) d[0] = f[0];
+        } else {
+            const bool in = !SLAB || (ez < 0 ? c >= k.plane : (ez > 0 ? c < k.last : true));
+            const uint32_t tf = in ? (BATCH ? tfl[I] : (uint32_t)fl2[c + off]) & 0x7fu : 0u;
+            if (tf == 0) { if (tgt_ok) d[(IX)I * k.ncx + off] = f[I]; }
+            else if (!own) {}
+            else if (tf == 1) d[(IX)D3Q19<I>::opp * k.ncx] = f[I];
+            else d[(IX)D3Q19<I>::opp * k.ncx] = Ar<T, E>::sub(f[I], T(p.lidc[I]));
+        }
+    };
+    [&]<int... Is>(std::integer_sequence<int, Is...>) { (push(std::integral_constant<int, Is>{}), ...); }
+    (std::make_integer_sequence<int, 19>{});
+}
+
+template <typename IX>
+__device__ __forceinline__ PushCtx<IX> push_ctx(const LbmParams& p, bool slab, int& pa, int& pb) {
+    PushCtx<IX> k;
+    k.plane = (size_t)p.nx * p.ny;
+    const size_t nc = k.plane * p.nzb;               // SoA stride of one population
+    pa = slab ? max(p.za - 1, 0) : p.za;
+    pb = slab ? min(p.zb + 1, p.nzb) : p.zb;
+    k.lo0 = (size_t)p.za * k.plane; k.lo1 = k.lo0 + k.plane;   // [lo0, lo1): plane za
+    k.hi1 = (size_t)p.zb * k.plane; k.hi0 = k.hi1 - k.plane;   // [hi0, hi1): plane zb-1
+    k.last = (size_t)(p.nzb - 1) * k.plane;
+    k.ncx = (IX)nc; k.pl = (IX)k.plane;
+    k.nx = p.nx;
+    return k;
+}
+
+// SLAB (Z-slab sweeps): output planes [za, zb) of a buffer with
+// ghost planes.  In push form a plane receives populations from its z
+// neighbours, so source planes [za-1, zb+1) are processed and only stores whose
+// target plane lies in [za, zb) are kept (each (cell, population) of the output
+// planes is still written exactly once).  Single-domain sweeps have no ghosts:
+// source and target ranges coincide and no store is filtered.
 template <typename T, bool E, typename IX, bool BATCH, bool SLAB>
 __global__ void __launch_bounds__(256, (BATCH ? 2 : 4))
 lbm_push_kernel(const T* __restrict__ src, T* __restrict__ dst, const uint8_t* __restrict__ fl2,
                 const LbmParams p) {
-    // SLAB (Z-slab sweeps): output planes [za, zb) of a buffer with
-    // ghost planes.  In push form a plane receives populations from its z
-    // neighbours, so source planes [za-1, zb+1) are processed and only stores whose
-    // target plane lies in [za, zb) are kept (each (cell, population) of the output
-    // planes is still written exactly once).  Single-domain sweeps have no ghosts:
-    // source and target ranges coincide and no store is filtered.
-    const size_t plane = (size_t)p.nx * p.ny;
-    const size_t nc = plane * p.nzb;              // SoA stride of one population
-    const int pa = SLAB ? max(p.za - 1, 0) : p.za, pb = SLAB ? min(p.zb + 1, p.nzb) : p.zb;
-    const size_t c0 = (size_t)pa * plane;
-    const size_t ncell = (size_t)(pb - pa) * plane;
-    const size_t lo0 = (size_t)p.za * plane, lo1 = lo0 + plane;       // [lo0, lo1): plane za
-    const size_t hi1 = (size_t)p.zb * plane, hi0 = hi1 - plane;       // [hi0, hi1): plane zb-1
-    const size_t last = (size_t)(p.nzb - 1) * plane;
+    int pa, pb;
+    const PushCtx<IX> k = push_ctx<IX>(p, SLAB, pa, pb);
+    const size_t c0 = (size_t)pa * k.plane;
+    const size_t ncell = (size_t)(pb - pa) * k.plane;
     const T omega = T(p.omega);
-    const int nx = p.nx;
-    const IX ncx = (IX)nc, pl = (IX)plane;   // 32-bit offsets when 19 populations fit (host choice)
     for (size_t t = blockIdx.x * (size_t)blockDim.x + threadIdx.x; t < ncell; t += (size_t)gridDim.x * blockDim.x) {
         const size_t c = c0 + t;
-        // SLAB: which stores reach an output plane (ez = -1 / 0 / +1 targets)
-        const bool own = !SLAB || (c >= lo0 && c < hi1);
-        const bool dn_ok = !SLAB || c >= lo1;     // target plane q-1 >= za
-        const bool up_ok = !SLAB || c < hi0;      // target plane q+1 < zb
         const uint32_t fl = fl2[c];
         const T* __restrict__ s = src + c;
         T f[19];
 #pragma unroll
-        for (int i = 0; i < 19; ++i) f[i] = s[(IX)i * ncx];
-        T* __restrict__ d = dst + c;
-        if (fl & 0x7fu) {   // WALL / LID: copied through
-            if (own) {
-#pragma unroll
-                for (int i = 0; i < 19; ++i) d[(IX)i * ncx] = f[i];
-            }
-            continue;
-        }
-        collide<T, E>(f, omega);
-        uint32_t tfl[19];
-        if constexpr (BATCH) {
-            auto ld = [&](auto Ic) {
-                constexpr int I = decltype(Ic)::value;
-                const IX off = (IX)D3Q19<I>::ex + (IX)D3Q19<I>::ey * (IX)nx + (IX)D3Q19<I>::ez * pl;
-                // (SLAB: a neighbour outside the buffer is never a store target; read nothing)
-                const bool in = !SLAB || (D3Q19<I>::ez < 0 ? c >= plane : (D3Q19<I>::ez > 0 ? c < last : true));
-                tfl[I] = (I == 0 || !in) ? 0u : (uint32_t)__ldg(fl2 + c + off);
-            };
-            [&]<int... Is>(std::integer_sequence<int, Is...>) { (ld(std::integral_constant<int, Is>{}), ...); }
-            (std::make_integer_sequence<int, 19>{});
-        }
-        auto push = [&](auto Ic) {
-            constexpr int I = decltype(Ic)::value;
-            constexpr int ez = D3Q19<I>::ez;
-            const IX off = (IX)D3Q19<I>::ex + (IX)D3Q19<I>::ey * (IX)nx + (IX)ez * pl;
-            const bool tgt_ok = ez < 0 ? dn_ok : (ez > 0 ? up_ok : own);
-            if constexpr (I == 0) {
-                if (own) d[0] = f[0];
-            } else {
-                const bool in = !SLAB || (ez < 0 ? c >= plane : (ez > 0 ? c < last : true));
-                const uint32_t tf = in ? (BATCH ? tfl[I] : (uint32_t)fl2[c + off]) & 0x7fu : 0u;
-                if (tf == 0) { if (tgt_ok) d[(IX)I * ncx + off] = f[I]; }
-                else if (!own) {}
-                else if (tf == 1) d[(IX)D3Q19<I>::opp * ncx] = f[I];
-                else d[(IX)D3Q19<I>::opp * ncx] = Ar<T, E>::sub(f[I], T(p.lidc[I]));
-            }
-        };
-        [&]<int... Is>(std::integer_sequence<int, Is...>) { (push(std::integral_constant<int, Is>{}), ...); }
-        (std::make_integer_sequence<int, 19>{});
+        for (int i = 0; i < 19; ++i) f[i] = s[(IX)i * k.ncx];
+        lbm_push_cell<T, E, IX, BATCH, SLAB>(f, fl, c, fl2, dst, k, omega, p);
     }
 }
 
