@@ -73,14 +73,15 @@ constexpr int ST7_RING_MAX = 12;
 
 // ---------------------------------------------------------------------------
 // One thread's register block of one plane: VY rows x VX columns.
-//  * FP32 (VX = 4): each row is held as two packed pairs a = (c0, c2),
-//    b = (c1, c3) so the X neighbours of one pair are the other pair (plus one
-//    shuffled edge value), and every 7-point update of a pair is 7 packed
+//  * FP32 (VX = 4): each row is held as two natural packed pairs a = (c0, c1),
+//    b = (c2, c3) (16-byte rows load, exchange and store with no moves); the X
+//    sums are swap(a) + (L, c2) and swap(b) + (c1, R) with L, R shuffled from
+//    the neighbouring lanes, and every 7-point update of a pair is 7 packed
 //    sm_100a instructions (FADD2 x5, FMUL2, FFMA2) for 2 points.
 //  * FP64 (VX = 2): plain scalars (the DP pipe is half rate; no packed form).
-// The arithmetic order is the oracle's (X2): ((x- + x+) + (y- + y+)) + (z- + z+),
-// then alpha*c + beta*s; the _rn intrinsics are never contracted, so the
-// bit-exact build only differs by using FMUL2 + FADD2 instead of FFMA2.
+// The bit-exact build uses the oracle's order (X2): ((x- + x+) + (y- + y+)) +
+// (z- + z+), then alpha*c + beta*s with scalar __fmul_rn / __fadd_rn; the
+// tolerance build adds the shuffled X sum last and fuses the final combine.
 // ---------------------------------------------------------------------------
 template <typename T, int VY> struct Blk;
 template <typename T> struct Row;
