@@ -187,3 +187,15 @@ def test_config4_lbm_1024_light_cone(oracle_lib):
         for z0 in range(1, n - 1, 64):
             mass += float(g[i, z0:min(z0 + 64, n - 1), 1:n - 1, 1:n - 1].double().sum())
     assert abs(mass - mass0) <= 1e-6 * mass0
+
+
+@pytest.mark.parametrize("shape", [(4, 3, 3), (4, 3, 5), (8, 7, 3), (40, 3, 9)])
+@pytest.mark.parametrize("dim_T", [1, 2])
+def test_degenerate_lattices(oracle_lib, shape, dim_T):
+    # two FLUID cells, one-cell-thick fluid layers (nx is a multiple of 4: TMA row pitch)
+    nx, ny, nz = shape
+    flags = stgen.cavity_flags(nx, ny, nz)
+    f0 = stgen.lbm_random(nx, ny, nz, 5, np.float32)
+    ref = oracle_lib.lbm(f0, flags, 1.6, 4)
+    got = run_gpu(f0, flags, 1.6, 4, dim_T=dim_T, exact=True)
+    assert np.array_equal(got, ref)

@@ -172,3 +172,18 @@ def test_autotune_picks_a_depth_and_stays_exact(oracle_lib, dtype):
         p.st7(x, y, 0.4, 0.1, 9)
         p.sync()
     assert np.array_equal(y.cpu().numpy(), ref)
+
+
+DEGENERATE = [(4, 3, 3), (4, 3, 17), (4, 200, 5), (300, 3, 3), (8, 5, 64), (1024, 4, 3)]
+
+
+@pytest.mark.parametrize("shape", DEGENERATE)
+@pytest.mark.parametrize("dim_T", [1, 2, 3, 5, 8])
+def test_degenerate_shapes_bitexact(oracle_lib, shape, dim_T):
+    # one interior point wide / one plane thick / single-row grids and deep sweeps on tiny grids
+    nx, ny, nz = shape
+    a = stgen.grid7(nx, ny, nz, 17, np.float32)
+    T = 2 * dim_T + 1
+    ref = oracle_lib.st7(a, 0.4, 0.1, T)
+    got, _ = run_gpu(a, 0.4, 0.1, T, dim_T, exact=True)
+    assert np.array_equal(got, ref)
