@@ -388,11 +388,15 @@ static bool overlap(const void* a, const void* b, size_t n) {
 // work items, in tile-major order, are cut into G contiguous ranges of equal
 // COST, where a range pays its planes plus a fixed overhead per tile segment it
 // touches (the 2*dim_T prolog/epilog rounds that fill and drain the on-chip
-// levels, at about half a steady round each, plus the first plane's load
-// latency).  Minimises the largest cost by bisection over a greedy cut.
+// levels, which run only some levels, plus the first plane's load latency;
+// calibrated by measurement below).  Minimises the largest cost by bisection
+// over a greedy cut.
 static void split_work(int ntiles, int nzo, int d, int G, int* split) {
     const long long work = (long long)ntiles * nzo;
-    const long long ovh = d + 2;
+    // measured on B200 (ST_SPLIT_OVH A/B, 256^3): 4 plane-equivalents per segment is
+    // best at dim_T 3 and 4 (+2 % over the d + 2 model); shallower sweeps restart cheaper
+    long long ovh = std::min(d + 1, 4);
+    if (const char* e = getenv("ST_SPLIT_OVH")) ovh = std::max(1, atoi(e));   // A/B tuning
     auto cuts = [&](long long C, int* out) {   // CTAs needed with per-CTA cost cap C
         if (C <= ovh) return G + 1;             // no CTA could take a plane
         long long it = 0;
