@@ -174,7 +174,7 @@ def cpu_baseline_7pt(n):
     oracle.st7(a, 0.4, 0.1, Ts)
     dt = time.perf_counter() - t0
     if dt < 6.0:   # the 8-sweep probe is dominated by per-call overhead: rescale once to ~12 s
-        Ts = int(max(1, min(20000, round(Ts * 12.0 / max(dt, 1e-3)))))
+        Ts = int(max(1, min(20000, 4 * Ts, round(Ts * 12.0 / max(dt, 1e-3)))))
         t0 = time.perf_counter()
         oracle.st7(a, 0.4, 0.1, Ts)
         dt = time.perf_counter() - t0
