@@ -161,26 +161,23 @@ def run_reference(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
-def cpu_baseline_7pt(n):
-    """the oracle timed on a bounded sample (~10 s) of the headline workload."""
+def cpu_baseline_7pt(n, T):
+    """the oracle timed on a bounded sample (~12 s) of the headline workload: whole
+    configs[1] runs (T sweeps of the n^3 grid), as many as fit."""
     import oracle
     import stgen
     a = stgen.grid7(n, n, n, 2, np.float32)
     t0 = time.perf_counter()
-    oracle.st7(a, 0.4, 0.1, 8)
-    t1 = (time.perf_counter() - t0) / 8          # per sweep (incl. the oracle's own copies)
-    Ts = int(max(1, min(20000, round(12.0 / max(t1, 1e-4)))))
+    oracle.st7(a, 0.4, 0.1, T)
+    t1 = time.perf_counter() - t0
+    reps = int(max(1, min(200, round(12.0 / max(t1, 1e-3)))))
     t0 = time.perf_counter()
-    oracle.st7(a, 0.4, 0.1, Ts)
+    for _ in range(reps):
+        oracle.st7(a, 0.4, 0.1, T)
     dt = time.perf_counter() - t0
-    if dt < 6.0:   # the 8-sweep probe is dominated by per-call overhead: rescale once to ~12 s
-        Ts = int(max(1, min(20000, 4 * Ts, round(Ts * 12.0 / max(dt, 1e-3)))))
-        t0 = time.perf_counter()
-        oracle.st7(a, 0.4, 0.1, Ts)
-        dt = time.perf_counter() - t0
-    return {"value": round((n - 2) ** 3 * Ts / dt / 1e6, 2), "unit": "Mupdates/s",
+    return {"value": round((n - 2) ** 3 * T * reps / dt / 1e6, 2), "unit": "Mupdates/s",
             "cores": oracle.num_threads(), "kind": "oracle",
-            "sample": f"7-point FP32 {n}^3, T={Ts} sweeps ({dt:.1f} s), OpenMP over z"}
+            "sample": f"7-point FP32 {n}^3, {reps} runs of T={T} ({dt:.1f} s), OpenMP over z"}
 
 
 # ----------------------------------------------------------------------------
@@ -435,7 +432,7 @@ def main():
                                                        "unit": "GB/s", "frac": round(gbs / hbm_gbs, 4)}}
             del fa, fb, flb
             torch.cuda.empty_cache()
-    cpu = cpu_baseline_7pt(n) if (rank == 0 and world == 1) else None
+    cpu = cpu_baseline_7pt(n, T) if (rank == 0 and world == 1) else None
 
     if rank == 0:
         line = {
