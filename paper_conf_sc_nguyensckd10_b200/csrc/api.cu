@@ -878,8 +878,9 @@ static int launch_lbm(st_plan* p, const void* src, void* dst, const uint8_t* fla
     const int pa = sv.single ? sv.za : std::max(sv.za - 1, 0), pb = sv.single ? sv.zb : std::min(sv.zb + 1, sv.nzb);
     const long long cells = (long long)(pb - pa) * p->nx * p->ny;
     if (cells <= 0 || sv.zb <= sv.za) return ST_OK;
-    // one wave of resident 256-thread CTAs (launch bounds: 4 per SM, 2 for the batched-flag kernel), grid-stride
-    int bps = lbm_push_batched((int)esize(p->dtype), p->nx, p->ny, sv.nzb) ? 2 : 4;
+    // one wave of resident 256-thread CTAs (the kernel's launch bounds), grid-stride
+    const bool batched = lbm_push_batched((int)esize(p->dtype), p->nx, p->ny, sv.nzb);
+    int bps = p->dtype == ST_F32 ? lbm_push_ctas<float>(batched) : lbm_push_ctas<double>(batched);
     if (const char* e = getenv("ST_LBM_BPS")) bps = std::max(1, atoi(e));   // A/B tuning
     const int grid = (int)std::min<long long>((cells + 255) / 256, (long long)p->sms * bps);
     cudaError_t e = lbm_push_launch(p->dtype == ST_F32 ? 0 : 1, p->exact, !sv.single, src, dst, sv.fl2, prm, grid,

@@ -4,12 +4,11 @@
 
 namespace st35d {
 
-// FP32 lattices of more than 2^24 cells run the batched-flag kernel at 2
-// CTAs/SM: it holds 23-27 GLUPS from 320^3 to 1024^3 (22.7 vs 15.4 at 1024^3,
-// 22.9 vs 18.5 at 512^3, 26.6 vs 20.2 at 448^3), while the per-direction
-// kernel at 4 CTAs/SM swings with the lattice size and is 3 % faster only up to
-// 256^3 (tools/lbm_big.py, T = 20); FP64 always batches.  ST_LBM_BATCH=0/1
-// overrides (A/B).
+// FP32 lattices of more than 2^24 cells run the batched-flag kernel (3 CTAs/SM):
+// it holds 25-28 GLUPS from 320^3 to 1024^3 (25.4 vs 15.4 at 1024^3, 25.6 vs
+// 18.5 at 512^3), while the per-direction kernel at 4 CTAs/SM swings with the
+// lattice size and only matches it up to 256^3 (tools/lbm_big.py, T = 20);
+// FP64 always batches (2 CTAs/SM).  ST_LBM_BATCH=0/1 overrides (A/B).
 bool lbm_push_batched(int esize, int nx, int ny, int nzb) {
     if (const char* e = getenv("ST_LBM_BATCH")) return atoi(e) != 0;
     return esize == 8 || (long long)nx * ny * nzb > (1LL << 24);

@@ -221,8 +221,12 @@ __device__ __forceinline__ PushCtx<IX> push_ctx(const LbmParams& p, bool slab, i
 // target plane lies in [za, zb) are kept (each (cell, population) of the output
 // planes is still written exactly once).  Single-domain sweeps have no ghosts:
 // source and target ranges coincide and no store is filtered.
+// CTAs per SM: per-direction flags 4 (64 registers); batched flags 3 for FP32
+// (80 registers) and 2 for FP64 (128 registers), all without spills
+template <typename T> constexpr int lbm_push_ctas(bool batch) { return batch ? (sizeof(T) == 4 ? 3 : 2) : 4; }
+
 template <typename T, bool E, typename IX, bool BATCH, bool SLAB>
-__global__ void __launch_bounds__(256, (BATCH ? 2 : 4))
+__global__ void __launch_bounds__(256, lbm_push_ctas<T>(BATCH))
 lbm_push_kernel(const T* __restrict__ src, T* __restrict__ dst, const uint8_t* __restrict__ fl2,
                 const LbmParams p) {
     int pa, pb;
