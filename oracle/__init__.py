@@ -42,6 +42,10 @@ def lib():
             fn.argtypes = [P, P, ctypes.c_long, ctypes.c_long, ctypes.c_long,
                            ctypes.c_double, ctypes.c_double, ctypes.c_int]
             fn.restype = ctypes.c_int
+            fn = getattr(L, f"oracle_st27_{sfx}")
+            fn.argtypes = [P, P, ctypes.c_long, ctypes.c_long, ctypes.c_long] + [ctypes.c_double] * 4 + \
+                [ctypes.c_int]
+            fn.restype = ctypes.c_int
             fn = getattr(L, f"oracle_lbm_{sfx}")
             fn.argtypes = [P, P, P, ctypes.c_long, ctypes.c_long, ctypes.c_long,
                            ctypes.c_double, ctypes.c_int, ctypes.c_double, ctypes.c_double,
@@ -75,6 +79,18 @@ def st7(A0: np.ndarray, alpha: float, beta: float, T: int) -> np.ndarray:
         A0.ctypes.data, out.ctypes.data, nx, ny, nz, alpha, beta, T)
     if rc != 0:
         raise RuntimeError(f"oracle_st7 rc={rc}")
+    return out
+
+
+def st27(A0: np.ndarray, alpha: float, beta: float, gamma: float, delta: float, T: int) -> np.ndarray:
+    """T Jacobi sweeps of the 27-point stencil (weights centre/face/edge/corner), Dirichlet shell."""
+    A0 = np.ascontiguousarray(A0)
+    nz, ny, nx = A0.shape
+    out = np.empty_like(A0)
+    rc = getattr(lib(), f"oracle_st27_{_sfx(A0.dtype)}")(
+        A0.ctypes.data, out.ctypes.data, nx, ny, nz, alpha, beta, gamma, delta, T)
+    if rc != 0:
+        raise RuntimeError(f"oracle_st27 rc={rc}")
     return out
 
 

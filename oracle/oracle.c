@@ -79,6 +79,81 @@ DEFINE_ST7(float, f32)
 DEFINE_ST7(double, f64)
 
 /* ------------------------------------------------------------------------ */
+/* 27-point stencil: the 3x3x3 cube around the      */
+/* centre; "the edge points, corners and face neighbors are multiplied by    */
+/* different constants", "4 multiplies, 26 adds":                            */
+/*   B = alpha*C + beta*F + gamma*E + delta*K                                */
+/* C centre, F the 6 face neighbours (one offset non-zero), E the 12 edge    */
+/* points (two offsets non-zero), K the 8 corners (three non-zero).          */
+/* Same Jacobi sweep / swap and fixed shell (X1) as the 7-point.      */
+/* Summation order (reading X24; the paper gives none): with, for plane      */
+/* z+dz,  v(dx) = a[dx,-1,dz] + a[dx,+1,dz]   (the y pair of column dx),     */
+/*        h     = a[-1,0,dz]  + a[+1,0,dz]    (the x pair),                  */
+/*        f(dz) = h + v(0)       (the 4 in-plane face points of plane dz),   */
+/*        e(dz) = v(-1) + v(+1)  (the 4 in-plane corner points of plane dz), */
+/*   F = f(0) + (a[0,0,-1] + a[0,0,+1])                                      */
+/*   E = e(0) + (f(-1) + f(+1))                                              */
+/*   K = e(-1) + e(+1)                                                       */
+/*   B = ((alpha*C + beta*F) + gamma*E) + delta*K                            */
+/* Each of the 26 neighbours enters exactly once: 4+2 / 4+4+4 / 4+4, and    */
+/* there are 26 additions (F 5, E 11, K 7, final 3) and 4 products, as      */
+/* P:119 counts.  F has the 7-point order of X2; every pair is symmetric,   */
+/* so x, y and z mirrors are bit-exact.                                      */
+/* ------------------------------------------------------------------------ */
+#define DEFINE_ST27(TYPE, SUFFIX)                                                     \
+static TYPE st27_f_##SUFFIX(const TYPE* a, long nx, long ny, long x, long y, long z)  \
+{                                                                                     \
+    TYPE h = a[IDX(x - 1, y, z)] + a[IDX(x + 1, y, z)];                               \
+    TYPE v = a[IDX(x, y - 1, z)] + a[IDX(x, y + 1, z)];                               \
+    return h + v;                                                                     \
+}                                                                                     \
+static TYPE st27_e_##SUFFIX(const TYPE* a, long nx, long ny, long x, long y, long z)  \
+{                                                                                     \
+    TYPE vm = a[IDX(x - 1, y - 1, z)] + a[IDX(x - 1, y + 1, z)];                      \
+    TYPE vp = a[IDX(x + 1, y - 1, z)] + a[IDX(x + 1, y + 1, z)];                      \
+    return vm + vp;                                                                   \
+}                                                                                     \
+int oracle_st27_##SUFFIX(const TYPE* A0, TYPE* out, long nx, long ny, long nz,        \
+                         double alpha_d, double beta_d, double gamma_d,               \
+                         double delta_d, int T)                                       \
+{                                                                                     \
+    if (nx < 1 || ny < 1 || nz < 1 || T < 0) return -1;                               \
+    const size_t n = (size_t)nx * ny * nz;                                            \
+    const TYPE alpha = (TYPE)alpha_d, beta = (TYPE)beta_d;   /* X19 */                \
+    const TYPE gamma = (TYPE)gamma_d, delta = (TYPE)delta_d;                          \
+    TYPE* a = (TYPE*)malloc(n * sizeof(TYPE));                                        \
+    TYPE* b = (TYPE*)malloc(n * sizeof(TYPE));                                        \
+    if (!a || !b) { free(a); free(b); return -2; }                                    \
+    memcpy(a, A0, n * sizeof(TYPE));                                                  \
+    memcpy(b, A0, n * sizeof(TYPE));                                                  \
+    for (int t = 0; t < T; ++t) {                                                     \
+        _Pragma("omp parallel for schedule(static)")                                  \
+        for (long z = 1; z < nz - 1; ++z)                                             \
+            for (long y = 1; y < ny - 1; ++y)                                         \
+                for (long x = 1; x < nx - 1; ++x) {                                   \
+                    TYPE zc = a[IDX(x, y, z - 1)] + a[IDX(x, y, z + 1)];              \
+                    TYPE F = st27_f_##SUFFIX(a, nx, ny, x, y, z) + zc;                \
+                    TYPE E = st27_e_##SUFFIX(a, nx, ny, x, y, z)                      \
+                             + (st27_f_##SUFFIX(a, nx, ny, x, y, z - 1)               \
+                                + st27_f_##SUFFIX(a, nx, ny, x, y, z + 1));           \
+                    TYPE K = st27_e_##SUFFIX(a, nx, ny, x, y, z - 1)                  \
+                             + st27_e_##SUFFIX(a, nx, ny, x, y, z + 1);               \
+                    TYPE p = alpha * a[IDX(x, y, z)];                                 \
+                    TYPE q = beta * F;                                                \
+                    TYPE r = gamma * E;                                               \
+                    TYPE s = delta * K;                                               \
+                    b[IDX(x, y, z)] = ((p + q) + r) + s;                              \
+                }                                                                     \
+        TYPE* tmp = a; a = b; b = tmp;                                                \
+    }                                                                                 \
+    memcpy(out, a, n * sizeof(TYPE));                                                 \
+    free(a); free(b);                                                                 \
+    return 0;                                                                         \
+}
+DEFINE_ST27(float, f32)
+DEFINE_ST27(double, f64)
+
+/* ------------------------------------------------------------------------ */
 /* D3Q19 lattice Boltzmann, push form (X13):                     */
 /*   1. read the 19 values of the cell and its flag           */
 /*   2. compute new values: BGK collision (X9)                               */
