@@ -36,6 +36,7 @@ TRAFFIC_PATH = os.path.join(ROOT, "profiles", "traffic.json")
 SM_COUNT = 148
 FP32_LANES, FP64_LANES = 128, 64
 ST7_OPS = 7            # FP instructions per 7-point update: 5 add, 1 mul, 1 fma (8 flops)
+ST27_OPS = 16          # FP instructions per 27-point update in the plane-factorised order X24: 12 add + 4 mul
 LBM_BYTES = {4: 153, 8: 305}   # (19*2*E + 1) per LBM update at dim_T = 1 (X12)
 
 
@@ -354,6 +355,29 @@ def main():
                                  "dim_T": D5, "dim_T_sweep": sw5, "ms_per_step": round(ms5, 3),
                                  "frac_alu": round(ST7_OPS * upd5 / (ms5 / 1e3) / (ops_peak * 1e12), 4),
                                  "info": inf5}
+        # 27-point stencil on the configs[1] grid, T = 100, every depth
+        for dtn, dt_np, tdt, dmax, lanes in (("f32", np.float32, torch.float32, 4, 128),
+                                             ("f64", np.float64, torch.float64, 2, FP64_LANES)):
+            x27 = torch.from_numpy(stgen.grid7(n, n, n, 2, dt_np)).cuda()
+            y27 = torch.empty_like(x27)
+            sw27, l27 = {}, 0
+            for d in range(1, dmax + 1):
+                with st.Plan(n, n, n, tdt, d) as p27:
+                    p27.set_stream(stream)
+                    t27, _ = time_steps(lambda: p27.st27(x27, y27, 0.3, 0.05, 0.02, 0.01, T), 2, 1)
+                    sw27[d] = round((n - 2) ** 3 * T / (t27 / 2 / 1e3) / 1e6, 1)
+                    l27 = max(l27, p27.last_launches())
+            d27 = max(sw27, key=sw27.get)
+            v27 = sw27[d27] * 1e6
+            E27 = 4 if dtn == "f32" else 8
+            extras[f"st27_{dtn}_256"] = {
+                "value": sw27[d27], "unit": "Mupdates/s", "dim_T": d27, "dim_T_sweep": sw27,
+                "roofline_hbm": {"achieved": round(2 * E27 / d27 * v27 / 1e9, 1), "peak": hbm_gbs, "unit": "GB/s",
+                                 "frac": round(2 * E27 / d27 * v27 / 1e9 / hbm_gbs, 4)},
+                "frac_alu": round(ST27_OPS * v27 / (SM_COUNT * lanes * sm_max * 1e6), 4),
+                "note": f"{ST27_OPS} FP instructions per update (plane-factorised order X24, no FMA); "
+                        "the paper's definition counts 30 (4 mul + 26 add, P:119)"}
+            del x27, y27
         # ablation ladder (Fig. 5(b)): no blocking -> 2.5D (dim_T = 1)
         # -> 3.5D (measured dim_T), same grid and T; plus the eq. (3) model's dim_T seed (f3)
         xa = torch.from_numpy(stgen.grid7(n, n, n, 2, np.float32)).cuda()

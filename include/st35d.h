@@ -88,6 +88,21 @@ st_plan* st_plan_create(int nx, int ny, int nz, st_dtype dtype, int dim_T);
 int st7_run(st_plan* plan, const void* in, void* out, double alpha, double beta, int T);
 
 /*
+ * st27_run — out = A(T): T Jacobi sweeps of the 27-point stencil (P:119,
+ * SURVEY §8(f) f1): "the edge points, corners and face neighbors are
+ * multiplied by different constants",
+ *     B = alpha*C + beta*(6 faces) + gamma*(12 edges) + delta*(8 corners)
+ * over the 3x3x3 cube of every interior point; the shell is fixed as for
+ * st7_run.  Summation order: DESIGN.md reading X24 (bit-identical to the
+ * oracle with st_plan_set_bitexact(plan, 1), FMA-contracted otherwise).
+ * Sweeps of depth min(dim_T, 4 FP32 / 2 FP64) are kept on chip (3.5D).  Same
+ * buffers, ownership (`in` is scratch), pointer kinds (device: asynchronous
+ * on the plan stream; host: staged and synchronous) and errors as st7_run.
+ * Single process only: ST_EUNSUPPORTED after st_plan_set_dist.
+ */
+int st27_run(st_plan* plan, const void* in, void* out, double alpha, double beta, double gamma, double delta, int T);
+
+/*
  * lbm_d3q19_run — f_dst = state after T D3Q19 steps of f_src,
  * BGK single-relaxation collision with relaxation rate omega (0 <= omega < 2;
  * omega = 0 is pure streaming), push semantics: the stored state is

@@ -740,6 +740,56 @@ extern "C" int st7_run(st_plan* p, const void* in, void* out, double alpha, doub
 }
 
 // ----------------------------------------------------------------------------
+// 27-point stencil: ceil(T/D) ping-pong sweeps of the
+// st27.cu kernel, D = min(dim_T, st27_depth_max()); single process only.
+// ----------------------------------------------------------------------------
+static int run27_device(st_plan* p, const void* in, void* out, const double w[4], int T) {
+    const size_t n = (size_t)p->nx * p->ny * p->nz * esize(p->dtype);
+    p->launches = 0;
+    if (T == 0) {
+        CUDA_TRY(cudaMemcpyAsync(out, in, n, cudaMemcpyDeviceToDevice, p->stream));
+        return ST_OK;
+    }
+    const int D = std::min(p->dimT, st27_depth_max(p->dtype == ST_F32 ? 0 : 1));
+    const std::vector<int> ds = sweep_depths(T, D);
+    void* bufs[2] = {const_cast<void*>(in), out};
+    for (size_t k = 0; k < ds.size(); ++k) {
+        cudaError_t e = st27_launch(p->dtype == ST_F32 ? 0 : 1, p->exact, ds[k], bufs[k % 2], bufs[(k + 1) % 2], p->nx,
+                                    p->ny, p->nz, w[0], w[1], w[2], w[3], p->sms, p->stream, nullptr);
+        if (e != cudaSuccess) return fail(ST_ECUDA, "st27 launch: %s", cudaGetErrorString(e));
+        ++p->launches;
+    }
+    if (ds.size() % 2 == 0) CUDA_TRY(cudaMemcpyAsync(out, in, n, cudaMemcpyDeviceToDevice, p->stream));
+    return ST_OK;
+}
+
+extern "C" int st27_run(st_plan* p, const void* in, void* out, double alpha, double beta, double gamma, double delta,
+                        int T) {
+    if (!p) return fail(ST_EINVAL, "NULL plan");
+    if (!in || !out) return fail(ST_EINVAL, "NULL grid pointer");
+    if (T < 0) return fail(ST_EINVAL, "T = %d < 0", T);
+    if (p->dist.mode != Dist::SINGLE) return fail(ST_EUNSUPPORTED, "st27_run is single-process only");
+    const size_t n = (size_t)p->nx * p->ny * p->nz * esize(p->dtype);
+    if (overlap(in, out, n)) return fail(ST_EINVAL, "in and out overlap");
+    const int kin = ptr_kind(in), kout = ptr_kind(out);
+    if (kin != kout) return fail(ST_EINVAL, "in and out must both be host or both be device pointers");
+    const double w[4] = {alpha, beta, gamma, delta};
+    if (kin == 1) {
+        if ((reinterpret_cast<uintptr_t>(in) | reinterpret_cast<uintptr_t>(out)) & 15)
+            return fail(ST_EINVAL, "device grids must be 16-byte aligned");
+        return run27_device(p, in, out, w, T);
+    }
+    int rc = ensure_hbuf(p, n);
+    if (rc) return rc;
+    CUDA_TRY(cudaMemcpyAsync(p->hbuf[0], in, n, cudaMemcpyHostToDevice, p->stream));
+    rc = run27_device(p, p->hbuf[0], p->hbuf[1], w, T);
+    if (rc) return rc;
+    CUDA_TRY(cudaMemcpyAsync(out, p->hbuf[1], n, cudaMemcpyDeviceToHost, p->stream));
+    CUDA_TRY(cudaStreamSynchronize(p->stream));
+    return ST_OK;
+}
+
+// ----------------------------------------------------------------------------
 // Blocking-parameter selection by measurement ("a framework that
 // determines the various blocking parameters"): the eq. (3) bound eta from this
 // device's HBM bandwidth and FP issue rate seeds the report; every depth

@@ -55,4 +55,9 @@ cudaError_t lbm_shell_check(const uint8_t* flags, int nx, int ny, int nz, int* d
 
 constexpr int ST7_MAXT = 256;
 
+// 27-point 3.5D sweep (st27.cu), depth D in [1, st27_depth_max()]; grid_out = CTAs launched
+int st27_depth_max(int dtype);
+cudaError_t st27_launch(int dtype, bool exact, int D, const void* in, void* out, int nx, int ny, int nz, double alpha,
+                        double beta, double gamma, double delta, int sms, cudaStream_t s, int* grid_out);
+
 }  // namespace st35d
