@@ -3,8 +3,11 @@
 // cube (centre, 6 faces, 12 edges, 8 corners), Jacobi two-grid sweeps,
 // Dirichlet shell (X1), dim_T levels kept on chip.
 //
-// Mapping (B200, sm_100a).  One CTA = a 32 x 32 loaded XY tile (16 warps of
-// 32 lanes x 2 rows) streamed along a Z chunk.  The 27-point sum factorises
+// Mapping (B200, sm_100a).  One CTA = a 32 x 32 loaded XY tile (8 warps of
+// 32 lanes x 4 rows FP32, 32 x 16 with 2 rows FP64) streamed along a Z chunk,
+// two CTAs per SM (<= 128 registers) so one CTA's barrier waits overlap the
+// other's work (measured at 256^3 FP32 dim_T 2: 16 warps x 2 rows 329, x 4
+// rows 351, 8 warps x 4 rows 408, x 8 rows 247 Gupd/s).  The 27-point sum factorises
 // by plane (reading X24): for every plane of a level each point forms
 //   v = a[y-1] + a[y+1],  h = a[x-1] + a[x+1],  f = h + v,  e = v[x-1] + v[x+1]
 // once (x pairs by warp shuffle, the y neighbours of a warp's edge rows
@@ -45,10 +48,18 @@ template <typename T> struct Op<T, false> {
 };
 
 constexpr int TW = 32;       // loaded tile width (one warp)
-constexpr int TH = 32;       // loaded tile height
-constexpr int VY = 2;        // rows per thread
-constexpr int NWARP = TH / VY;
+#ifndef ST27_NWARP
+#define ST27_NWARP 8
+#endif
+constexpr int NWARP = ST27_NWARP;
 constexpr int NTHR = TW * NWARP;
+constexpr int MINB = 512 / NTHR;   // CTAs per SM at <= 128 registers
+#ifndef ST27_VY32
+#define ST27_VY32 4
+#endif
+// loaded tile height and rows per thread: FP32 64 rows (4 per thread), FP64 32 (2)
+template <typename T> constexpr int vy_of() { return sizeof(T) == 4 ? ST27_VY32 : 2; }
+template <typename T> constexpr int th_of() { return NWARP * vy_of<T>(); }
 }  // namespace
 
 struct St27Params {
@@ -57,8 +68,9 @@ struct St27Params {
 };
 
 template <typename T, int D, bool EX>
-__global__ void __launch_bounds__(NTHR, 1) st27_kernel(const T* __restrict__ a, T* __restrict__ b, St27Params p) {
+__global__ void __launch_bounds__(NTHR, MINB) st27_kernel(const T* __restrict__ a, T* __restrict__ b, St27Params p) {
     using O = Op<T, EX>;
+    constexpr int VY = vy_of<T>(), TH = th_of<T>();
     __shared__ T sm[2][TH][TW];
     const int lane = threadIdx.x, w = threadIdx.y;
     const int tiles = p.ntx * p.nty;
@@ -94,7 +106,7 @@ __global__ void __launch_bounds__(NTHR, 1) st27_kernel(const T* __restrict__ a, 
     // ring (each thread copies and later reads only its own VY elements, so no
     // barrier guards the ring; the loads stay in flight across the rounds'
     // barriers instead of stalling every round on HBM latency)
-    constexpr int PF = sizeof(T) == 4 ? 6 : 3;
+    constexpr int PF = 3;
     __shared__ T ring[PF][TH][TW];
     auto issue = [&](int pl, int slot) {
         const size_t pb = (size_t)min(pl, hi0 - 1) * plane;
@@ -222,7 +234,7 @@ static int choose_chunks(int ntiles, int nz, int D, int slots) {
     return (nz + best - 1) / best;
 }
 
-// FP64 at D >= 3 spills under the 128-register cap of a 512-thread CTA
+// FP64 at D >= 3 spills under the 128-register cap (FP32 D = 4 spills too, kept for the sweep)
 int st27_depth_max(int dtype) { return dtype == 0 ? 4 : 2; }
 
 cudaError_t st27_launch(int dtype, bool exact, int D, const void* in, void* out, int nx, int ny, int nz, double alpha,
@@ -231,6 +243,7 @@ cudaError_t st27_launch(int dtype, bool exact, int D, const void* in, void* out,
     St27Params p;
     p.nx = nx; p.ny = ny; p.nz = nz;
     p.ntx = nx <= TW ? 1 : 1 + (nx - TW + (TW - 2 * D) - 1) / (TW - 2 * D);
+    const int TH = dtype == 0 ? th_of<float>() : th_of<double>();
     p.nty = ny <= TH ? 1 : 1 + (ny - TH + (TH - 2 * D) - 1) / (TH - 2 * D);
     p.zchunk = 0;
     if (dtype == 0) { p.alpha = (float)alpha; p.beta = (float)beta; p.gamma = (float)gamma; p.delta = (float)delta; }
