@@ -122,8 +122,9 @@ __global__ void __launch_bounds__(NTHR, MINB) st27_kernel(const T* __restrict__ 
 
     // one round with compile-time window rotation R: slot (R+2)%3 receives the
     // new plane, (R+1)%3 holds the middle, R%3 the lowest
-    auto round = [&](int i, auto Rc) {
+    auto round = [&](int i, auto Rc, auto Sc) {
         constexpr int R = decltype(Rc)::value;
+        constexpr bool SHELL = decltype(Sc)::value;           // false: no shell point in this round
         constexpr int sN = (R + 2) % 3, sC = (R + 1) % 3, sM = R % 3;
         T v[VY];
         issue(lo0 + i + PF - 1, (i + PF - 1) % PF);            // slot of plane i-1, already read
@@ -144,7 +145,8 @@ __global__ void __launch_bounds__(NTHR, MINB) st27_kernel(const T* __restrict__ 
                     const T K = O::add(we[L - 1][sM][j], we[L - 1][sN][j]);
                     const T r = O::add(O::add(O::add(O::mul(alpha, c0), O::mul(beta, F)), O::mul(gamma, E)),
                                        O::mul(delta, K));
-                    v[j] = (shxy[j] || shz) ? c0 : r;
+                    if constexpr (SHELL) v[j] = (shxy[j] || shz) ? c0 : r;
+                    else v[j] = r;
                 }
             }
             if (L == D) {                                       // final level: store the tile interior
@@ -178,11 +180,23 @@ __global__ void __launch_bounds__(NTHR, MINB) st27_kernel(const T* __restrict__ 
     };
     // rotation chosen per round (a loop body unrolled by three rounds gave
     // wrong results for the fourth round with this nvcc)
+    // (CTA-uniform) rounds of tiles off the XY shell whose levels' planes miss
+    // z = 0 and z = nz-1 take a body without the per-point shell select
+    const bool tile_shell = x0 == 0 || x0 + TW >= p.nx || y0 == 0 || y0 + TH >= p.ny;
+    using S1 = std::true_type;
+    using S0 = std::false_type;
     for (int i = 0; i < nround; ++i) {
         const int r = i % 3;
-        if (r == 0) round(i, std::integral_constant<int, 0>{});
-        else if (r == 1) round(i, std::integral_constant<int, 1>{});
-        else round(i, std::integral_constant<int, 2>{});
+        const bool sh = tile_shell || lo0 + i - D <= 0 || lo0 + i - 1 >= p.nz - 1;
+        if (sh) {
+            if (r == 0) round(i, std::integral_constant<int, 0>{}, S1{});
+            else if (r == 1) round(i, std::integral_constant<int, 1>{}, S1{});
+            else round(i, std::integral_constant<int, 2>{}, S1{});
+        } else {
+            if (r == 0) round(i, std::integral_constant<int, 0>{}, S0{});
+            else if (r == 1) round(i, std::integral_constant<int, 1>{}, S0{});
+            else round(i, std::integral_constant<int, 2>{}, S0{});
+        }
     }
 }
 
