@@ -58,7 +58,10 @@ constexpr int MINB = 512 / NTHR;   // CTAs per SM at <= 128 registers
 #define ST27_VY32 4
 #endif
 // loaded tile height and rows per thread: FP32 64 rows (4 per thread), FP64 32 (2)
-template <typename T> constexpr int vy_of() { return sizeof(T) == 4 ? ST27_VY32 : 2; }
+#ifndef ST27_VY64
+#define ST27_VY64 2
+#endif
+template <typename T> constexpr int vy_of() { return sizeof(T) == 4 ? ST27_VY32 : ST27_VY64; }
 template <typename T> constexpr int th_of() { return NWARP * vy_of<T>(); }
 }  // namespace
 
