@@ -9,7 +9,9 @@ store, sweep driver).  value = interior updates per second over all ranks
 (Mupdates/s; X3: an update is one interior point advanced one time step).
 
 Extra lines inside the same JSON object: FP64 256^3, FP32 512^3 (configs[3]
-per-GPU size) and the D3Q19 cavity 256^3 (configs[2], MLUPS).
+per-GPU size), the 27-point stencil FP32/FP64 256^3 at every depth (SURVEY
+f1), the ablation ladder and the D3Q19 cavity 256^3 / 1024^3 (configs[2],
+configs[4] lattice, MLUPS).
 
 Timing: W warm-up steps, then K steps each bracketed by CUDA events on the
 plan's stream; L2 (126 MB) is flushed by writing a 512 MiB buffer between
