@@ -111,16 +111,24 @@ __global__ void __launch_bounds__(NTHR, MINB) st27_kernel(const T* __restrict__ 
     // barriers instead of stalling every round on HBM latency)
     constexpr int PF = 3;
     __shared__ T ring[PF][TH][TW];
-    auto issue = [&](int pl, int slot) {
-        const size_t pb = (size_t)min(pl, hi0 - 1) * plane;
+    const T* gnext = a + (size_t)lo0 * plane;                  // next level-0 plane to copy
+    int pnext = lo0;
+    uint32_t off32[VY];
+#pragma unroll
+    for (int j = 0; j < VY; ++j) off32[j] = (uint32_t)off[j];
+    const uint32_t ring0 = smem_u32(&ring[0][w * VY][lane]);
+    auto issue = [&](int slot) {
 #pragma unroll
         for (int j = 0; j < VY; ++j)
-            asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" ::"r"(smem_u32(&ring[slot][w * VY + j][lane])),
-                         "l"(a + pb + off[j]), "n"(sizeof(T)) : "memory");
+            asm volatile("cp.async.ca.shared.global [%0], [%1], %2;"
+                         ::"r"(ring0 + (uint32_t)((slot * TH + j) * TW * sizeof(T))), "l"(gnext + off32[j]),
+                         "n"(sizeof(T)) : "memory");
         asm volatile("cp.async.commit_group;" ::: "memory");
+        if (pnext < hi0 - 1) { gnext += plane; ++pnext; }    // past the chunk: re-copy the last plane
     };
 #pragma unroll
-    for (int k = 0; k < PF - 1; ++k) issue(lo0 + k, k);
+    for (int k = 0; k < PF - 1; ++k) issue(k);
+    int rslot = 0;                                             // ring slot of this round's plane
     int buf = 0;
 
     // one round with compile-time window rotation R: slot (R+2)%3 receives the
@@ -130,10 +138,11 @@ __global__ void __launch_bounds__(NTHR, MINB) st27_kernel(const T* __restrict__ 
         constexpr bool SHELL = decltype(Sc)::value;           // false: no shell point in this round
         constexpr int sN = (R + 2) % 3, sC = (R + 1) % 3, sM = R % 3;
         T v[VY];
-        issue(lo0 + i + PF - 1, (i + PF - 1) % PF);            // slot of plane i-1, already read
+        issue(rslot == 0 ? PF - 1 : rslot - 1);                // slot of plane i-1, already read
         asm volatile("cp.async.wait_group %0;" ::"n"(PF - 1) : "memory");
 #pragma unroll
-        for (int j = 0; j < VY; ++j) v[j] = ring[i % PF][w * VY + j][lane];
+        for (int j = 0; j < VY; ++j) v[j] = ring[rslot][w * VY + j][lane];
+        rslot = rslot == PF - 1 ? 0 : rslot + 1;
 #pragma unroll
         for (int L = 0; L <= D; ++L) {
             const int q = lo0 + i - L;                          // plane of level L this round
@@ -154,9 +163,10 @@ __global__ void __launch_bounds__(NTHR, MINB) st27_kernel(const T* __restrict__ 
             }
             if (L == D) {                                       // final level: store the tile interior
                 if (q >= zs && q < ze) {
+                    T* ob = b + (size_t)q * plane;
 #pragma unroll
                     for (int j = 0; j < VY; ++j)
-                        if (st[j]) b[(size_t)q * plane + off[j]] = v[j];
+                        if (st[j]) ob[off32[j]] = v[j];
                 }
                 break;
             }
@@ -257,6 +267,7 @@ int st27_depth_max(int dtype) { return dtype == 0 ? 4 : 2; }
 cudaError_t st27_launch(int dtype, bool exact, int D, const void* in, void* out, int nx, int ny, int nz, double alpha,
                         double beta, double gamma, double delta, int sms, cudaStream_t s, int* grid_out) {
     if (D < 1 || D > st27_depth_max(dtype)) return cudaErrorInvalidValue;
+    if ((size_t)nx * ny >= (size_t(1) << 32)) return cudaErrorInvalidValue;   // 32-bit in-plane offsets
     St27Params p;
     p.nx = nx; p.ny = ny; p.nz = nz;
     p.ntx = nx <= TW ? 1 : 1 + (nx - TW + (TW - 2 * D) - 1) / (TW - 2 * D);
