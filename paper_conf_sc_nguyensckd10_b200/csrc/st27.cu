@@ -109,7 +109,10 @@ __global__ void __launch_bounds__(NTHR, MINB) st27_kernel(const T* __restrict__ 
     // ring (each thread copies and later reads only its own VY elements, so no
     // barrier guards the ring; the loads stay in flight across the rounds'
     // barriers instead of stalling every round on HBM latency)
-    constexpr int PF = 3;
+#ifndef ST27_PF
+#define ST27_PF 3
+#endif
+    constexpr int PF = ST27_PF;
     __shared__ T ring[PF][TH][TW];
     const T* gnext = a + (size_t)lo0 * plane;                  // next level-0 plane to copy
     int pnext = lo0;
