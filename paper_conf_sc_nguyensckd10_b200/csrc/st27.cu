@@ -57,7 +57,7 @@ constexpr int MINB = 512 / NTHR;   // CTAs per SM at <= 128 registers
 #ifndef ST27_VY32
 #define ST27_VY32 4
 #endif
-// loaded tile height and rows per thread: FP32 64 rows (4 per thread), FP64 32 (2)
+// loaded tile height = NWARP x rows per thread: FP32 32 (4 per thread), FP64 16 (2)
 #ifndef ST27_VY64
 #define ST27_VY64 2
 #endif
