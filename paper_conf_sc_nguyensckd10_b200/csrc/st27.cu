@@ -194,8 +194,9 @@ __global__ void __launch_bounds__(NTHR, MINB) st27_kernel(const T* __restrict__ 
             }
         }
     };
-    // rotation chosen per round (a loop body unrolled by three rounds gave
-    // wrong results for the fourth round with this nvcc)
+    // rotation chosen per round: the same three bodies called in sequence
+    // from a loop stepping by three rounds gave wrong values from the fourth
+    // round on (cause not isolated)
     // (CTA-uniform) rounds of tiles off the XY shell whose levels' planes miss
     // z = 0 and z = nz-1 take a body without the per-point shell select
     const bool tile_shell = x0 == 0 || x0 + TW >= p.nx || y0 == 0 || y0 + TH >= p.ny;
