@@ -147,6 +147,23 @@ int st_plan_set_bitexact(st_plan* plan, int on);
 enum { ST_VARIANT_35D = 0, ST_VARIANT_NAIVE = 1 };
 int st_plan_set_variant(st_plan* plan, int variant);
 
+/* Tuning and test selections (no environment variables are read).
+ *   ST_OPT_LBM_BATCHED  -1 (default) auto: FP32 lattices above 2^24 cells use the
+ *                       batched-flag push kernel; 0 / 1 force the per-direction /
+ *                       batched kernel (FP64 always batches).
+ *   ST_OPT_LBM_KERNEL   0 (default) auto: dim_T = 1 push kernel when the plan's LBM
+ *                       depth is 1, else the multi-level on-chip kernel; 1 push
+ *                       (dim_T = 1 sweeps); 2 multi-level kernel at the plan depth.
+ *   ST_OPT_OVERLAP      1 (default): Z-slab ghost exchange overlapped with the
+ *                       interior sweep on a side stream; 0 serialised.
+ *   ST_OPT_PDL          1 (default): 7-point sweeps chained with programmatic
+ *                       dependent launch; 0 plain launches.
+ *   ST_OPT_ST7_VARIANT  0 (default) auto; else VY*1000 + threads per CTA of a
+ *                       compiled 7-point kernel variant (4256, 4384, 2256).
+ * Results do not depend on any option.  Unknown option or value: ST_EINVAL. */
+enum { ST_OPT_LBM_BATCHED = 1, ST_OPT_LBM_KERNEL = 2, ST_OPT_OVERLAP = 3, ST_OPT_PDL = 4, ST_OPT_ST7_VARIANT = 5 };
+int st_plan_set_option(st_plan* plan, int option, int value);
+
 /* st_plan_autotune — choose the 7-point sweep depth by measurement (the
  * paper's "framework that determines the various blocking parameters", P:377,
  * eqs. (1)-(4) of §V-C).  Every depth 1..(deepest the plan tiles, <= dim_T)

@@ -21,6 +21,7 @@ ST_F32, ST_F64 = 0, 1
 ST_OK, ST_EINVAL, ST_ENOMEM, ST_ECUDA, ST_ENCCL, ST_EUNSUPPORTED = 0, -1, -2, -3, -4, -5
 ST_FLUID, ST_WALL, ST_LID = 0, 1, 2
 ST_MAX_DIM_T = 8
+ST_OPT_LBM_BATCHED, ST_OPT_LBM_KERNEL, ST_OPT_OVERLAP, ST_OPT_PDL, ST_OPT_ST7_VARIANT = 1, 2, 3, 4, 5
 _ERRNAMES = {-1: "ST_EINVAL", -2: "ST_ENOMEM", -3: "ST_ECUDA", -4: "ST_ENCCL", -5: "ST_EUNSUPPORTED"}
 
 
@@ -46,7 +47,7 @@ class st_blocking(ctypes.Structure):
 _lib = None
 
 EXPORTS = ["st_plan_create", "st7_run", "st27_run", "lbm_d3q19_run", "st_destroy", "st_last_error", "st_last_status",
-           "st_plan_set_stream", "st_plan_set_lbm_lid", "st_plan_set_bitexact", "st_plan_set_variant", "st_plan_autotune", "st_plan_sync",
+           "st_plan_set_stream", "st_plan_set_option", "st_plan_set_lbm_lid", "st_plan_set_bitexact", "st_plan_set_variant", "st_plan_autotune", "st_plan_sync",
            "st_plan_set_dist", "st_plan_set_loopback_slabs", "st_plan_ghost_planes", "st_plan_local_slab",
            "st_plan_get_info", "st_plan_last_launches", "st_blocking_model", "st_fig3_step",
            "st_nccl_unique_id", "st_slab_range"]
@@ -71,6 +72,7 @@ def lib() -> ctypes.CDLL:
         "st_last_status": ([], I),
         "st_plan_set_stream": ([P, P], I),
         "st_plan_set_lbm_lid": ([P, D, D, D], I),
+        "st_plan_set_option": ([P, I, I], I),
         "st_plan_set_bitexact": ([P, I], I),
         "st_plan_set_variant": ([P, I], I),
         "st_plan_autotune": ([P, P, P, I, ctypes.POINTER(I), ctypes.POINTER(ctypes.c_float)], I),
@@ -87,6 +89,8 @@ def lib() -> ctypes.CDLL:
         "st_slab_range": ([I, I, I, ctypes.POINTER(I), ctypes.POINTER(I)], I),
     }
     for name, (args, res) in sig.items():
+        if os.environ.get("ST35D_LIB") and not hasattr(L, name):   # A/B build of an older ABI
+            continue
         fn = getattr(L, name)
         fn.argtypes = args
         fn.restype = res
@@ -152,6 +156,11 @@ def st_plan_set_stream(plan: int, stream) -> int:
 
 def st_plan_set_lbm_lid(plan: int, ux: float, uy: float, uz: float) -> int:
     return _check(lib().st_plan_set_lbm_lid(plan, ux, uy, uz))
+
+
+def st_plan_set_option(plan: int, option: int, value: int) -> int:
+    """ST_OPT_* tuning / test selections (include/st35d.h); results do not depend on them."""
+    return _check(lib().st_plan_set_option(plan, int(option), int(value)))
 
 
 def st_plan_set_bitexact(plan: int, on: bool) -> int:
@@ -241,21 +250,84 @@ def dtype_code(dtype) -> int:
     raise ValueError(f"unsupported dtype {dtype}")
 
 
+def _buf_info(buf):
+    """(is_device, element size, dtype code or None, numel) of a tensor / array."""
+    if hasattr(buf, "data_ptr"):   # torch tensor
+        dev = buf.device.type == "cuda"
+        name = str(buf.dtype)
+        return dev, buf.element_size(), name, buf.numel()
+    if hasattr(buf, "ctypes"):     # numpy array
+        return False, buf.itemsize, str(buf.dtype), buf.size
+    return None
+
+
 class Plan:
-    """RAII wrapper: ``with Plan(nx, ny, nz, dtype, dim_T) as p: p.st7(a, b, ...)``."""
+    """RAII wrapper: ``with Plan(nx, ny, nz, dtype, dim_T) as p: p.st7(a, b, ...)``.
+
+    The methods check each tensor / array against the plan (device or host,
+    dtype, element count) before calling the C ABI, which only sees pointers
+    and could not detect a short or mistyped buffer (ValueError on mismatch).
+    Raw integer addresses are passed through unchecked."""
 
     def __init__(self, nx: int, ny: int, nz: int, dtype, dim_T: int):
-        self.h = st_plan_create(nx, ny, nz, dtype if isinstance(dtype, int) else dtype_code(dtype), dim_T)
+        self.dtype = dtype if isinstance(dtype, int) else dtype_code(dtype)
+        self.h = st_plan_create(nx, ny, nz, self.dtype, dim_T)
         self.shape = (nz, ny, nx)
+        self._nzb = nz
+
+    def _local_cells(self) -> int:
+        nz, ny, nx = self.shape
+        return nx * ny * self._nzb
+
+    def _check_bufs(self, bufs, ncomp: int, what: str) -> None:
+        want = "float32" if self.dtype == ST_F32 else "float64"
+        need = ncomp * self._local_cells()
+        kinds = set()
+        for b in bufs:
+            info = _buf_info(b)
+            if info is None:
+                continue
+            dev, _, name, n = info
+            kinds.add(dev)
+            if want not in name:
+                raise ValueError(f"{what}: buffer dtype {name} does not match the plan ({want})")
+            if n != need:
+                raise ValueError(f"{what}: buffer has {n} elements, the plan needs {need}")
+        if len(kinds) > 1:
+            raise ValueError(f"{what}: buffers must all be on the device or all on the host")
+
+    def _check_flags(self, flags, ref) -> None:
+        info = _buf_info(flags)
+        if info is None:
+            return
+        dev, esz, name, n = info
+        if "uint8" not in name:
+            raise ValueError(f"flags must be uint8, got {name}")
+        if n != self._local_cells():
+            raise ValueError(f"flags have {n} elements, the plan needs {self._local_cells()}")
+        r = _buf_info(ref)
+        if r is not None and r[0] != dev:
+            raise ValueError("flags and populations must both be on the device or both on the host")
 
     def st7(self, inp, out, alpha: float, beta: float, T: int) -> None:
+        self._check_bufs((inp, out), 1, "st7")
         st7_run(self.h, inp, out, alpha, beta, T)
 
     def st27(self, inp, out, alpha: float, beta: float, gamma: float, delta: float, T: int) -> None:
+        self._check_bufs((inp, out), 1, "st27")
         st27_run(self.h, inp, out, alpha, beta, gamma, delta, T)
 
     def lbm(self, f_src, f_dst, omega: float, T: int, flags) -> None:
+        self._check_bufs((f_src, f_dst), 19, "lbm")
+        self._check_flags(flags, f_src)
         lbm_d3q19_run(self.h, f_src, f_dst, omega, T, flags)
+
+    def set_option(self, option: int, value: int) -> None:
+        st_plan_set_option(self.h, option, value)
+
+    def set_dist(self, unique_id: bytes, rank: int, nranks: int) -> None:
+        st_plan_set_dist(self.h, unique_id, rank, nranks)
+        self._nzb = self.shape[0] if nranks == 1 else st_plan_local_slab(self.h)[1] + 2 * st_plan_ghost_planes(self.h)
 
     def set_stream(self, stream) -> None:
         st_plan_set_stream(self.h, stream)

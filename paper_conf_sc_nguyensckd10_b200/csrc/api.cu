@@ -67,7 +67,6 @@ static int encode_3d(CUtensorMap* map, const void* base, st_dtype dt, int nx, in
     // L2 promotion: the tile boxes start at arbitrary 16-byte offsets, so a
     // 256-byte promotion would fetch up to twice the requested sectors
     CUtensorMapL2promotion promo = CU_TENSOR_MAP_L2_PROMOTION_NONE;
-    if (const char* e = getenv("ST_L2PROMO")) promo = (CUtensorMapL2promotion)atoi(e);
     CUresult r = enc(map, dt == ST_F32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3,
                      const_cast<void*>(base), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
                      CU_TENSOR_MAP_SWIZZLE_NONE, promo, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
@@ -80,8 +79,10 @@ static int encode_3d(CUtensorMap* map, const void* base, st_dtype dt, int nx, in
 // ----------------------------------------------------------------------------
 struct Geo7 {
     int d = 0, VY = 0, NTX = 0, VX = 0, TX = 0, NTY = 0, TY = 0;
-    int hx = 0, wx = 0, wy = 0, tiles_x = 0, tiles_y = 0, threads = 0, grid = 0, maxt = 0, ring = 4;
-    bool split = false;   // warp-specialised two-group kernel (st7_split.cuh)
+    int hx = 0, wx = 0, wy = 0, tiles_x = 0, tiles_y = 0, threads = 0, grid = 0, ring = 0;
+    int ey = 0, ly_last = 0, oy0_last = 0;   // y placement (St7Params)
+    int maxt = 0;                            // threads of the kernel variant (>= threads launched)
+    int minb = 1;                            // CTAs per SM of the variant
     size_t smem = 0;
     double kappa = 0;
     St7LaunchFn fn = nullptr;
@@ -95,12 +96,19 @@ struct st_plan {
     int dimKmax = 0;   // deepest sweep the 7-point kernels can tile (<= dimT)
     int dev = 0, sms = 0;
     size_t smem_optin = 0;
+    size_t smem_sm = 0;        // shared memory per SM
     cudaStream_t stream = nullptr;
     bool own_stream = false;
     bool exact = false;
     int variant = ST_VARIANT_35D;    // st_plan_set_variant (ablation baseline ST_VARIANT_NAIVE)
     double lid[3] = {0.05, 0.0, 0.0};
     int launches = 0;
+    // st_plan_set_option (include/st35d.h): tuning / test selections, no environment variables
+    int opt_lbm_batched = -1;   // -1 auto
+    int opt_lbm_kernel = 0;     // 0 auto, 1 push, 2 multi-level
+    int opt_overlap = 1;
+    int opt_pdl = 1;
+    int opt_st7_variant = 0;    // 0 auto, else VY * 1000 + threads per CTA
     // host-pointer staging
     void* hbuf[2] = {nullptr, nullptr};
     size_t hbuf_bytes = 0;
@@ -120,41 +128,35 @@ static size_t esize(st_dtype d) { return d == ST_F32 ? 4 : 8; }
 struct GeoL { int TY = 0, wx = 0, wy = 0, tiles_x = 0, tiles_y = 0; size_t smem = 0; };
 static int planL(const st_plan* p, int d, GeoL& g);
 static int max_lbm_depth(const st_plan* p);
+static bool lbm_use_push(const st_plan* p);
 
-// Kernel variant (rows per thread VY, max threads per CTA) for a sweep depth:
-// the register budget of each (D, VY, MAXT) instantiation, from ptxas -v
-// (no spills): 512 threads cap registers at 128 and double the resident
-// warps; 256 threads allow 255 registers for the deeper Z windows.
-static void variant_for(st_dtype dt, int d, int& vy, int& maxt, bool& split) {
-    split = false;
-    if (const char* e = getenv("ST_VARIANT")) {  // "VYxMAXT[s]", e.g. 4x256, 4x512s (tuning only)
-        int a = 0, b = 0;
-        char c = 0;
-        const int n = sscanf(e, "%dx%d%c", &a, &b, &c);
-        if (n >= 2) { vy = a; maxt = b; split = n == 3 && c == 's' && d >= 2 && d <= 6; return; }
+// Kernel variant (rows per thread VY, threads per CTA) for a sweep depth.
+// Registers (ptxas -v) cap what fits: VY = 4 keeps 2 planes x 16 points per
+// level in registers and fits 256 threads up to dim_T = 4 without spills;
+// deeper sweeps use VY = 2 (half the window per thread, twice the exchange
+// traffic per point).  ST_OPT_ST7_VARIANT overrides (A/B).
+static void variant_for(const st_plan* p, int d, int& vy, int& nt, int& minb) {
+    minb = 1;
+    if (p->opt_st7_variant) {
+        vy = p->opt_st7_variant / 1000 % 10; nt = p->opt_st7_variant % 1000; minb = std::max(1, p->opt_st7_variant / 10000);
+        return;
     }
-    // measured on B200 (tools/quickbench.py): VY=4 / 256 threads is fastest
-    // while it fits without spills; deeper sweeps need the smaller block
-    if (dt == ST_F32) { vy = d <= 4 ? 4 : 2; maxt = 256; return; }
-    vy = d <= 3 ? 4 : 2; maxt = 256;
+    vy = d <= 4 ? 4 : 2;
+    nt = 256;
+    // FP64 (2 doubles per 16-byte vector, 32 threads per tile row): VY = 2 gives
+    // 16-row tiles, too short for dim_T >= 7 (written rows 16 - 2 dim_T)
+    if (p->dtype == ST_F64) vy = (d <= 3 || d >= 7) ? 4 : 2;
 }
 
-static St7LaunchFn lookup7(st_dtype dt, bool exact, int d, int vy, int maxt, bool split) {
-    if (split) {
-        if (dt == ST_F32) return exact ? st7s_lookup_f32_exact(d, vy, maxt) : st7s_lookup_f32_fast(d, vy, maxt);
-        return exact ? st7s_lookup_f64_exact(d, vy, maxt) : st7s_lookup_f64_fast(d, vy, maxt);
-    }
-    if (dt == ST_F32) return exact ? st7_lookup_f32_exact(d, vy, maxt) : st7_lookup_f32_fast(d, vy, maxt);
-    return exact ? st7_lookup_f64_exact(d, vy, maxt) : st7_lookup_f64_fast(d, vy, maxt);
+static St7LaunchFn lookup7(st_dtype dt, bool exact, int d, int vy, int nt, int minb) {
+    if (dt == ST_F32) return exact ? st7_lookup_f32_exact(d, vy, nt, minb) : st7_lookup_f32_fast(d, vy, nt, minb);
+    return exact ? st7_lookup_f64_exact(d, vy, nt, minb) : st7_lookup_f64_fast(d, vy, nt, minb);
 }
 
 static size_t smem7(const Geo7& g, st_dtype dt, int ring) {
-    if (g.split)   // TMA ring + 4-plane hand-off ring + exchange [D-2][2][2][MAXT/2] + mbarriers
-        return (size_t)(ring + 4) * g.TX * g.TY * esize(dt) + (size_t)(g.d > 2 ? g.d - 2 : 0) * 4 * (g.maxt / 2) * 16 +
-               ring * 8;
-    // TMA ring + row exchange [D-1][2][2][MAXT] x 16 B + mbarriers
-    return (size_t)ring * g.TX * g.TY * esize(dt) + (size_t)(g.d > 1 ? g.d - 1 : 0) * 4 * g.maxt * 16 +
-           ring * 8;
+    // TMA ring + row exchange [D-1][2][2][threads] x 16 B + mbarriers + load cursor
+    return (size_t)ring * g.TX * g.TY * esize(dt) + (size_t)(g.d > 1 ? g.d - 1 : 0) * 4 * g.threads * 16 +
+           ST7_RING_MAX * 8;
 }
 
 // Planner for one sweep depth d over an nx x ny plane with nzo output planes:
@@ -162,53 +164,66 @@ static size_t smem7(const Geo7& g, st_dtype dt, int ring) {
 // shared memory for the TMA ring and the Y exchange), then the XY tile that
 // minimises computed points per plane (halo + ragged last tile), then a
 // persistent grid of one CTA per SM with equal (tile, z) volume per CTA.
+// y placement of a tile height (see st7_tile in st7_kernel.cuh): the regular
+// tiles are shifted down by ey so that y = 0 is the last row of a thread's
+// block, the last tile is placed so that y = ny-1 is the first row of a block;
+// no halo is needed beyond a grid face (the shell is fixed), so the first and
+// last tiles write up to the face
+static void place_y(Geo7& g, int ny, int d) {
+    g.wy = g.TY - 2 * d;
+    g.ey = ((g.VY - 1 - d) % g.VY + g.VY) % g.VY;
+    g.ly_last = g.oy0_last = 0;
+    if (g.TY - d - g.ey >= ny) { g.tiles_y = 1; return; }
+    g.ly_last = ny - 1 - (g.TY - g.VY);
+    g.oy0_last = std::max(g.ly_last + d, 0);
+    g.tiles_y = std::max(1, (g.oy0_last + g.ey + g.wy - 1) / g.wy) + 1;
+}
+
 static int plan7(st_plan* p, int d, int nzo, Geo7& g) {
     g.d = d;
     g.VX = p->dtype == ST_F32 ? 4 : 2;
     g.NTX = p->dtype == ST_F32 ? 16 : 32;
     g.TX = g.NTX * g.VX;
-    variant_for(p->dtype, d, g.VY, g.maxt, g.split);
+    int ntmax = 0;
+    variant_for(p, d, g.VY, ntmax, g.minb);
     g.hx = (d + g.VX - 1) / g.VX * g.VX;
     g.wx = (g.TX - g.hx - d) & ~(g.VX - 1);
-    if (g.wx < g.VX) return fail(ST_EUNSUPPORTED, "dim_T %d too deep for a %d-wide tile", d, g.TX);
+    if (g.wx < g.VX) return fail(ST_EUNSUPPORTED, "dim_T %d too deep for the %d-wide tile of this build", d, g.TX);
     g.tiles_x = (p->nx + g.wx - 1) / g.wx;
-    const int ntymax = g.maxt / (g.split ? 2 : 1) / g.NTX;   // thread rows per (group of the) CTA
+    // tile height: the thread-row count (<= the variant's threads) that loads
+    // the fewest rows per plane (tiles_y * TY); ties go to the taller tile
     long best = -1;
-    for (int nty = 2; nty <= ntymax; ++nty) {
-        if (g.split && (g.NTX * nty) % 32) continue;   // groups must be whole warps
+    for (int nty = 2; nty <= ntmax / g.NTX; ++nty) {
         Geo7 c = g;
         c.NTY = nty;
         c.TY = nty * c.VY;
-        c.threads = c.NTX * nty * (c.split ? 2 : 1);
-        c.wy = c.TY - 2 * d;
-        if (c.wy < 1) continue;
-        c.tiles_y = (p->ny + c.wy - 1) / c.wy;
-        // TMA ring: as deep as shared memory allows (prefetch ring-2 planes ahead:
-        // the plane loads must cover HBM latency, several rounds of compute)
+        c.threads = c.NTX * nty;
+        if (c.TY - 2 * d < 1) continue;
+        place_y(c, p->ny, d);
+        // TMA ring: as deep as shared memory allows (the loads run ring-2 planes
+        // ahead and must cover HBM latency, several rounds of compute)
         c.ring = 0;
-        for (int r = ST7_RING_MAX; r >= 5; --r)
-            if (smem7(c, p->dtype, r) <= p->smem_optin) { c.ring = r; break; }
-        if (const char* e = getenv("ST_RING")) c.ring = std::min(c.ring, atoi(e));
-        if (c.ring < 5) continue;
+        for (int r = ST7_RING_MAX; r >= 4; --r)
+            if (smem7(c, p->dtype, r) <= (g.minb == 1 ? p->smem_optin : p->smem_sm / g.minb - 1024)) { c.ring = r; break; }
+        if (c.ring < 4) continue;
         c.smem = smem7(c, p->dtype, c.ring);
-        long cost = (long)c.tiles_y * c.TY;
-        if (best < 0 || cost < best || (cost == best && c.TY > g.TY)) {
-            best = cost;
-            g = c;
-        }
+        const long cost = (long)c.tiles_y * c.TY;
+        if (best < 0 || cost < best || (cost == best && c.TY > g.TY)) { best = cost; g = c; }
     }
-    if (best < 0) return fail(ST_EUNSUPPORTED, "no tile fits dim_T %d", d);
+    if (best < 0) return fail(ST_EUNSUPPORTED, "dim_T %d too deep for the tiles of this build", d);
     const long long work = (long long)g.tiles_x * g.tiles_y * nzo;
-    g.grid = (int)std::min<long long>(p->sms, std::max<long long>(work, 1));
+    g.grid = (int)std::min<long long>((long long)p->sms * g.minb, std::max<long long>(work, 1));
     g.kappa = (double)g.tiles_x * g.TX * g.tiles_y * g.TY / ((double)p->nx * p->ny);
-    g.fn = lookup7(p->dtype, p->exact, d, g.VY, g.maxt, g.split);
-    if (!g.fn) return fail(ST_EUNSUPPORTED, "no kernel for dim_T %d", d);
+    g.fn = lookup7(p->dtype, p->exact, d, g.VY, ntmax, g.minb);
+    if (!g.fn) return fail(ST_EUNSUPPORTED, "no kernel for dim_T %d (VY %d, %d threads)", d, g.VY, ntmax);
+    g.maxt = ntmax;
     return ST_OK;
 }
 
 static int get_geo7(st_plan* p, int d, int nzo, Geo7*& out) {
     auto it = p->geo7.find(d);
-    if (it == p->geo7.end() || it->second.fn != lookup7(p->dtype, p->exact, d, it->second.VY, it->second.maxt, it->second.split)) {
+    if (it == p->geo7.end() ||
+        it->second.fn != lookup7(p->dtype, p->exact, d, it->second.VY, it->second.maxt, it->second.minb)) {
         Geo7 g;
         int rc = plan7(p, d, nzo, g);
         if (rc) return rc;
@@ -217,7 +232,7 @@ static int get_geo7(st_plan* p, int d, int nzo, Geo7*& out) {
     out = &it->second;
     // grid depends on the output-plane count of the call
     const long long work = (long long)out->tiles_x * out->tiles_y * nzo;
-    out->grid = (int)std::min<long long>(p->sms, std::max<long long>(work, 1));
+    out->grid = (int)std::min<long long>((long long)p->sms * out->minb, std::max<long long>(work, 1));
     return ST_OK;
 }
 
@@ -241,6 +256,7 @@ extern "C" st_plan* st_plan_create(int nx, int ny, int nz, st_dtype dtype, int d
     p->dev = dev;
     p->sms = prop.multiProcessorCount;
     p->smem_optin = prop.sharedMemPerBlockOptin;
+    p->smem_sm = prop.sharedMemPerMultiprocessor;
     if (cudaStreamCreateWithFlags(&p->stream, cudaStreamNonBlocking) != cudaSuccess) {
         fail(ST_ECUDA, "stream create"); delete p; return nullptr;
     }
@@ -249,12 +265,17 @@ extern "C" st_plan* st_plan_create(int nx, int ny, int nz, st_dtype dtype, int d
         fail(ST_ENOMEM, "scratch"); st_destroy(p); return nullptr;
     }
     p->dist.init_single(nz);
-    // deepest 7-point sweep that tiles on one SM (f64 at dim_T 7-8 does not:
-    // those plans run sweeps of depth dimK < dim_T; results are identical)
+    // the 7-point sweep of depth dim_T must tile (D > D_max is an
+    // error, not a silent shallower sweep)
     Geo7* g = nullptr;
-    for (int d = dim_T; d >= 1; --d)
-        if (get_geo7(p, d, nz, g) == ST_OK) { p->dimK = p->dimKmax = d; break; }
-    if (!p->dimK) { st_destroy(p); return nullptr; }
+    if (get_geo7(p, dim_T, nz, g) != ST_OK) {
+        const std::string msg = g_err;
+        const int code = g_code;
+        st_destroy(p);
+        fail(code, "%s", msg.c_str());
+        return nullptr;
+    }
+    p->dimK = p->dimKmax = dim_T;
     g_err.clear();
     g_code = 0;
     return p;
@@ -294,6 +315,27 @@ extern "C" int st_plan_set_variant(st_plan* p, int variant) {
     return ST_OK;
 }
 
+extern "C" int st_plan_set_option(st_plan* p, int option, int value) {
+    if (!p) return fail(ST_EINVAL, "NULL plan");
+    switch (option) {
+        case ST_OPT_LBM_BATCHED:
+            if (value < -1 || value > 1) return fail(ST_EINVAL, "ST_OPT_LBM_BATCHED %d", value);
+            p->opt_lbm_batched = value; return ST_OK;
+        case ST_OPT_LBM_KERNEL:
+            if (value < 0 || value > 2) return fail(ST_EINVAL, "ST_OPT_LBM_KERNEL %d", value);
+            p->opt_lbm_kernel = value; return ST_OK;
+        case ST_OPT_OVERLAP: p->opt_overlap = value != 0; return ST_OK;
+        case ST_OPT_PDL: p->opt_pdl = value != 0; return ST_OK;
+        case ST_OPT_ST7_VARIANT:
+            if (value != 0 && !lookup7(p->dtype, p->exact, 1, value / 1000 % 10, value % 1000, std::max(1, value / 10000)))
+                return fail(ST_EINVAL, "ST_OPT_ST7_VARIANT %d is not compiled", value);
+            p->opt_st7_variant = value;
+            p->geo7.clear();
+            return ST_OK;
+        default: return fail(ST_EINVAL, "unknown option %d", option);
+    }
+}
+
 extern "C" int st_plan_set_bitexact(st_plan* p, int on) {
     if (!p) return fail(ST_EINVAL, "NULL plan");
     p->exact = on != 0;
@@ -329,7 +371,7 @@ extern "C" int st_plan_get_info(const st_plan* p, int lbm, st_plan_info* info) {
         info->tiles_x = g.tiles_x; info->tiles_y = g.tiles_y; info->ctas = p->sms; info->threads = 32 * g.TY;
         info->smem_bytes = (int)g.smem;
         info->kappa = (double)g.tiles_x * 32 * g.tiles_y * g.TY / ((double)p->nx * p->ny);
-        info->kernel = (d == 1 && getenv("ST_LBM_35D") == nullptr) ? 100 : 200 + d;
+        info->kernel = lbm_use_push(p) ? 100 : 200 + d;
         info->dim_t_sweep = d;
         return ST_OK;
     }
@@ -339,7 +381,7 @@ extern "C" int st_plan_get_info(const st_plan* p, int lbm, st_plan_info* info) {
     const Geo7& g = *gp;
     info->tile_x = g.TX; info->tile_y = g.TY; info->out_x = g.wx; info->out_y = g.wy;
     info->tiles_x = g.tiles_x; info->tiles_y = g.tiles_y; info->ctas = g.grid; info->threads = g.threads;
-    info->smem_bytes = (int)g.smem; info->kappa = g.kappa; info->kernel = g.VY * 1000 + g.maxt + (g.split ? 100000 : 0);
+    info->smem_bytes = (int)g.smem; info->kappa = g.kappa; info->kernel = g.minb * 10000 + g.VY * 1000 + g.maxt;
     info->dim_t_sweep = p->dimK;
     info->ring = g.ring;
     return ST_OK;
@@ -395,8 +437,7 @@ static void split_work(int ntiles, int nzo, int d, int G, int* split) {
     const long long work = (long long)ntiles * nzo;
     // measured on B200 (ST_SPLIT_OVH A/B, 256^3): 4 plane-equivalents per segment is
     // best at dim_T 3 and 4 (+2 % over the d + 2 model); shallower sweeps restart cheaper
-    long long ovh = std::min(d + 1, 4);
-    if (const char* e = getenv("ST_SPLIT_OVH")) ovh = std::max(1, atoi(e));   // A/B tuning
+    const long long ovh = std::min(d + 1, 4);
     auto cuts = [&](long long C, int* out) {   // CTAs needed with per-CTA cost cap C
         if (C <= ovh) return G + 1;             // no CTA could take a plane
         long long it = 0;
@@ -438,31 +479,16 @@ static int launch7(st_plan* p, const void* src, void* dst, int d, double alpha, 
     prm.za = sv.za; prm.zb = sv.zb;
     prm.tiles_x = g->tiles_x; prm.ntiles = g->tiles_x * g->tiles_y;
     prm.wx = g->wx; prm.wy = g->wy; prm.hx = g->hx;
-    prm.work = (long long)prm.ntiles * (sv.zb - sv.za);
+    prm.tiles_y = g->tiles_y; prm.ey = g->ey; prm.ly_last = g->ly_last; prm.oy0_last = g->oy0_last;
     prm.ring = g->ring;
-    if (const char* e = getenv("ST_DBG")) prm.dbg = atoi(e);
+    prm.pdl = p->opt_pdl;
     prm.alpha = alpha; prm.beta = beta;
-    if (prm.work <= 0) return ST_OK;
+    if ((long long)prm.ntiles * (sv.zb - sv.za) <= 0) return ST_OK;
+    if ((long long)prm.ntiles * (sv.zb - sv.za) >= (1LL << 31)) return fail(ST_EUNSUPPORTED, "grid too large");
     const int grid = std::min(sv.grid_cap > 0 ? std::min(g->grid, sv.grid_cap) : g->grid, ST7_MAX_GRID);
     split_work(prm.ntiles, sv.zb - sv.za, d, grid, prm.split);
-    // tuning builds (-DST7_PROF=1): ST_PROF_OUT=file appends per-warp phase clocks of every launch
-    const char* prof_out = getenv("ST_PROF_OUT");
-    const size_t prof_n = (size_t)grid * 16 * 10;
-    if (prof_out && cudaMalloc(&prm.prof, prof_n * 8) == cudaSuccess) cudaMemset(prm.prof, 0, prof_n * 8);
     cudaError_t e = g->fn(&map, prm, grid, g->threads, g->smem, sv.stream ? sv.stream : p->stream);
     if (e != cudaSuccess) return fail(ST_ECUDA, "st7 launch (d=%d): %s", d, cudaGetErrorString(e));
-    if (prm.prof) {
-        std::vector<unsigned long long> h(prof_n);
-        cudaStreamSynchronize(sv.stream ? sv.stream : p->stream);
-        cudaMemcpy(h.data(), prm.prof, prof_n * 8, cudaMemcpyDeviceToHost);
-        cudaFree(prm.prof);
-        if (FILE* f = fopen(prof_out, "ab")) {
-            const int hdr[4] = {grid, g->maxt / 32, d, (int)(sv.zb - sv.za)};
-            fwrite(hdr, sizeof hdr, 1, f);
-            fwrite(h.data(), 8, prof_n, f);
-            fclose(f);
-        }
-    }
     ++p->launches;
     return ST_OK;
 }
@@ -585,13 +611,13 @@ static int ensure_comm(st_plan* p) {
 // the interior of sweep k: the d' output planes next to each
 // slab face are computed first, an event hands them to the exchange stream,
 // the interior planes are computed meanwhile, and sweep k+1 waits for the
-// exchange.  ST_NO_OVERLAP=1 serialises exchange and sweep (A/B tuning).
+// exchange.  ST_OPT_OVERLAP = 0 serialises exchange and sweep (A/B).
 template <typename L>
 static int run_sweeps(st_plan* p, const std::vector<int>& ds, const void* in, void* out, int ncomp,
                       const uint8_t* flags, L&& launch) {
     Dist& D = p->dist;
     const size_t pb = (size_t)p->nx * p->ny * esize(p->dtype);
-    const bool overlap_ok = getenv("ST_NO_OVERLAP") == nullptr;
+    const bool overlap_ok = p->opt_overlap != 0;
     if (D.mode == Dist::SINGLE) {
         const void* src = in;
         void* dst = out;
@@ -893,6 +919,12 @@ static int max_lbm_depth(const st_plan* p) {
     return 1;
 }
 
+static bool lbm_use_push(const st_plan* p) {
+    if (p->opt_lbm_kernel == 1) return true;
+    if (p->opt_lbm_kernel == 2) return false;
+    return max_lbm_depth(p) == 1;
+}
+
 static int launch_lbm35(st_plan* p, const void* src, void* dst, int d, double omega, const SlabView& sv) {
     GeoL g;
     int rc = planL(p, d, g);
@@ -929,12 +961,11 @@ static int launch_lbm(st_plan* p, const void* src, void* dst, const uint8_t* fla
     const long long cells = (long long)(pb - pa) * p->nx * p->ny;
     if (cells <= 0 || sv.zb <= sv.za) return ST_OK;
     // one wave of resident 256-thread CTAs (the kernel's launch bounds), grid-stride
-    const bool batched = lbm_push_batched((int)esize(p->dtype), p->nx, p->ny, sv.nzb);
-    int bps = p->dtype == ST_F32 ? lbm_push_ctas<float>(batched) : lbm_push_ctas<double>(batched);
-    if (const char* e = getenv("ST_LBM_BPS")) bps = std::max(1, atoi(e));   // A/B tuning
+    const bool batched = lbm_push_batched((int)esize(p->dtype), p->nx, p->ny, sv.nzb, p->opt_lbm_batched);
+    const int bps = p->dtype == ST_F32 ? lbm_push_ctas<float>(batched) : lbm_push_ctas<double>(batched);
     const int grid = (int)std::min<long long>((cells + 255) / 256, (long long)p->sms * bps);
-    cudaError_t e = lbm_push_launch(p->dtype == ST_F32 ? 0 : 1, p->exact, !sv.single, src, dst, sv.fl2, prm, grid,
-                                    sv.stream ? sv.stream : p->stream);
+    cudaError_t e = lbm_push_launch(p->dtype == ST_F32 ? 0 : 1, p->exact, !sv.single, batched, src, dst, sv.fl2, prm,
+                                    grid, sv.stream ? sv.stream : p->stream);
     if (e != cudaSuccess) return fail(ST_ECUDA, "lbm launch: %s", cudaGetErrorString(e));
     ++p->launches;
     return ST_OK;
@@ -963,8 +994,8 @@ static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T
         return ST_OK;
     }
     // dim_T = 1: the fused push kernel (fastest measured on B200); dim_T >= 2:
-    // the on-chip multi-level sweep lbm_35d (ST_LBM_35D=1 forces it for dim_T = 1)
-    const bool push = max_lbm_depth(p) == 1 && getenv("ST_LBM_35D") == nullptr;
+    // the on-chip multi-level sweep lbm_35d (ST_OPT_LBM_KERNEL selects either)
+    const bool push = lbm_use_push(p);
     // neighbour-flag prepass, every call (a reused flags pointer may hold new contents; ~1 pass over the flags)
     if (p->dist.mode != Dist::LOOPBACK) {
         const size_t cells = (size_t)p->nx * p->ny * p->dist.nzb;

@@ -11,10 +11,10 @@ namespace st35d {
 
 // launch with programmatic stream serialization (PDL): the kernel's prologue may
 // overlap the previous kernel in the stream; the kernel orders its memory
-// accesses after it with griddepcontrol.wait (ST_NO_PDL=1: plain launch, A/B)
+// accesses after it with griddepcontrol.wait (pdl = false: plain launch, ST_OPT_PDL A/B)
 template <typename K, typename... A>
-inline cudaError_t launch_pdl(K kernel, int grid, int threads, size_t smem, cudaStream_t s, A... args) {
-    static const bool off = getenv("ST_NO_PDL") != nullptr;
+inline cudaError_t launch_pdl(bool pdl, K kernel, int grid, int threads, size_t smem, cudaStream_t s, A... args) {
+    const bool off = !pdl;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(grid);
     cfg.blockDim = dim3(threads);
@@ -31,20 +31,15 @@ inline cudaError_t launch_pdl(K kernel, int grid, int threads, size_t smem, cuda
 using St7LaunchFn = cudaError_t (*)(const CUtensorMap* map, const St7Params& p, int grid, int threads,
                                     size_t smem, cudaStream_t s);
 
-// returns nullptr if (D, VY) is not compiled
-St7LaunchFn st7_lookup_f32_fast(int D, int VY, int MAXT);
-St7LaunchFn st7_lookup_f32_exact(int D, int VY, int MAXT);
-St7LaunchFn st7_lookup_f64_fast(int D, int VY, int MAXT);
-St7LaunchFn st7_lookup_f64_exact(int D, int VY, int MAXT);
-// warp-specialised two-group variant (st7_split.cuh), D in [2, 6]
-St7LaunchFn st7s_lookup_f32_fast(int D, int VY, int MAXT);
-St7LaunchFn st7s_lookup_f32_exact(int D, int VY, int MAXT);
-St7LaunchFn st7s_lookup_f64_fast(int D, int VY, int MAXT);
-St7LaunchFn st7s_lookup_f64_exact(int D, int VY, int MAXT);
+// returns nullptr if (D, VY, NT, MINB) is not compiled
+St7LaunchFn st7_lookup_f32_fast(int D, int VY, int NT, int MINB);
+St7LaunchFn st7_lookup_f32_exact(int D, int VY, int NT, int MINB);
+St7LaunchFn st7_lookup_f64_fast(int D, int VY, int NT, int MINB);
+St7LaunchFn st7_lookup_f64_exact(int D, int VY, int NT, int MINB);
 
-bool lbm_push_batched(int esize, int nx, int ny, int nzb);   // kernel choice (also sets the grid)
-cudaError_t lbm_push_launch(int dtype, bool exact, bool slab, const void* src, void* dst, const uint8_t* fl2,
-                            const LbmParams& p, int grid, cudaStream_t s);
+bool lbm_push_batched(int esize, int nx, int ny, int nzb, int force);   // kernel choice (also sets the grid)
+cudaError_t lbm_push_launch(int dtype, bool exact, bool slab, bool batched, const void* src, void* dst,
+                            const uint8_t* fl2, const LbmParams& p, int grid, cudaStream_t s);
 cudaError_t lbm35_launch(int dtype, bool exact, int D, const Lbm35Params& p, int grid, int threads, size_t smem,
                          cudaStream_t s);
 cudaError_t st7_naive_launch(int dtype, const void* in, void* out, int nx, int ny, int nz, double alpha,
@@ -52,8 +47,6 @@ cudaError_t st7_naive_launch(int dtype, const void* in, void* out, int nx, int n
 cudaError_t lbm_fl2(const uint8_t* flags, uint8_t* fl2, int nx, int ny, int nz, cudaStream_t s);
 constexpr int LBM35_MAX_D = 3;
 cudaError_t lbm_shell_check(const uint8_t* flags, int nx, int ny, int nz, int* d_count, cudaStream_t s);
-
-constexpr int ST7_MAXT = 256;
 
 // 27-point 3.5D sweep (st27.cu), depth D in [1, st27_depth_max()]; grid_out = CTAs launched
 int st27_depth_max(int dtype);

@@ -8,14 +8,15 @@ namespace st35d {
 // it holds 25-28 GLUPS from 320^3 to 1024^3 (25.4 vs 15.4 at 1024^3, 25.6 vs
 // 18.5 at 512^3), while the per-direction kernel at 4 CTAs/SM swings with the
 // lattice size and only matches it up to 256^3 (tools/lbm_big.py, T = 20);
-// FP64 always batches (2 CTAs/SM).  ST_LBM_BATCH=0/1 overrides (A/B).
-bool lbm_push_batched(int esize, int nx, int ny, int nzb) {
-    if (const char* e = getenv("ST_LBM_BATCH")) return atoi(e) != 0;
+// FP64 always batches (2 CTAs/SM).  force = 0/1 overrides (st_plan_set_option
+// ST_OPT_LBM_BATCHED, used by the parity tests to reach both kernels).
+bool lbm_push_batched(int esize, int nx, int ny, int nzb, int force) {
+    if (force >= 0) return force != 0 || esize == 8;
     return esize == 8 || (long long)nx * ny * nzb > (1LL << 24);
 }
 
 template <typename T, bool E, bool SLAB>
-static cudaError_t push_t(const void* src, void* dst, const uint8_t* fl2, const LbmParams& p, int grid,
+static cudaError_t push_t(bool batched, const void* src, void* dst, const uint8_t* fl2, const LbmParams& p, int grid,
                           cudaStream_t s) {
     // FP64: 32-bit element offsets when every population offset (and a plane step)
     // fits; FP32 keeps 64-bit offsets (measured 26.0 vs 23.6 GLUPS at 256^3, tools/lbm_ab.sh)
@@ -25,7 +26,7 @@ static cudaError_t push_t(const void* src, void* dst, const uint8_t* fl2, const 
     if (sizeof(T) == 8) {
         if (span < (1LL << 31)) lbm_push_kernel<T, E, int, true, SLAB><<<grid, 256, 0, s>>>(a, b, fl2, p);
         else lbm_push_kernel<T, E, long long, true, SLAB><<<grid, 256, 0, s>>>(a, b, fl2, p);
-    } else if (lbm_push_batched(4, p.nx, p.ny, p.nzb)) {
+    } else if (batched) {
         lbm_push_kernel<T, E, long long, true, SLAB><<<grid, 256, 0, s>>>(a, b, fl2, p);
     } else {
         lbm_push_kernel<T, E, long long, false, SLAB><<<grid, 256, 0, s>>>(a, b, fl2, p);
@@ -34,18 +35,19 @@ static cudaError_t push_t(const void* src, void* dst, const uint8_t* fl2, const 
 }
 
 template <typename T, bool E>
-static cudaError_t push_s(bool slab, const void* src, void* dst, const uint8_t* fl2, const LbmParams& p, int grid,
-                          cudaStream_t s) {
-    return slab ? push_t<T, E, true>(src, dst, fl2, p, grid, s) : push_t<T, E, false>(src, dst, fl2, p, grid, s);
+static cudaError_t push_s(bool slab, bool batched, const void* src, void* dst, const uint8_t* fl2, const LbmParams& p,
+                          int grid, cudaStream_t s) {
+    return slab ? push_t<T, E, true>(batched, src, dst, fl2, p, grid, s)
+                : push_t<T, E, false>(batched, src, dst, fl2, p, grid, s);
 }
 
-// fl2 = the lbm_fl2 prepass output of the flags
-cudaError_t lbm_push_launch(int dtype, bool exact, bool slab, const void* src, void* dst, const uint8_t* fl2,
-                            const LbmParams& p, int grid, cudaStream_t s) {
-    if (dtype == 0) return exact ? push_s<float, true>(slab, src, dst, fl2, p, grid, s)
-                                 : push_s<float, false>(slab, src, dst, fl2, p, grid, s);
-    return exact ? push_s<double, true>(slab, src, dst, fl2, p, grid, s)
-                 : push_s<double, false>(slab, src, dst, fl2, p, grid, s);
+// fl2 = the lbm_fl2 prepass output of the flags; batched = lbm_push_batched(...)
+cudaError_t lbm_push_launch(int dtype, bool exact, bool slab, bool batched, const void* src, void* dst,
+                            const uint8_t* fl2, const LbmParams& p, int grid, cudaStream_t s) {
+    if (dtype == 0) return exact ? push_s<float, true>(slab, batched, src, dst, fl2, p, grid, s)
+                                 : push_s<float, false>(slab, batched, src, dst, fl2, p, grid, s);
+    return exact ? push_s<double, true>(slab, batched, src, dst, fl2, p, grid, s)
+                 : push_s<double, false>(slab, batched, src, dst, fl2, p, grid, s);
 }
 
 template <typename T, int D, bool E>

@@ -1,7 +1,7 @@
-// st7_inst.cu — instantiates st7_35d_kernel for one (dtype, mode); compiled
-// once per combination with -DST_T=float|double -DST_EXACT=0|1.
+// st7_inst.cu — instantiates the 7-point sweep kernel (st7_kernel.cuh) for one
+// (dtype, mode); compiled once per combination with -DST_T=float|double
+// -DST_EXACT=0|1 (build.py).
 #include "launch.h"
-#include "st7_split.cuh"
 
 #ifndef ST_T
 #define ST_T float
@@ -26,50 +26,38 @@ namespace st35d {
 namespace ST_UNIT_NS {
 
 using TT = ST_T;
-constexpr int NTX = sizeof(TT) == 4 ? 16 : 32;
+constexpr int NTX = sizeof(TT) == 4 ? 16 : 32;   // threads across the 64-point tile row
 
-template <int D, int VY, int MAXT>
-cudaError_t launch(const CUtensorMap* map, const St7Params& p, int grid, int threads, size_t smem,
-                   cudaStream_t s) {
-    auto k = st7_35d_kernel<TT, D, NTX, VY, ST_EXACT != 0, MAXT>;
+template <int D, int VY, int NT, int MINB>
+cudaError_t launch(const CUtensorMap* map, const St7Params& p, int grid, int threads, size_t smem, cudaStream_t s) {
+    auto k = st7_35d_kernel<TT, D, NTX, VY, ST_EXACT != 0, NT, MINB>;
+    if (threads > NT || threads % NTX) return cudaErrorInvalidValue;
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    return launch_pdl(k, grid, threads, smem, s, *map, p);
+    return launch_pdl(p.pdl != 0, k, grid, threads, smem, s, *map, p);
 }
 
-template <int VY, int MAXT>
+template <int VY, int NT, int MINB = 1>
 St7LaunchFn pick(int D) {
     switch (D) {
-        case 1: return launch<1, VY, MAXT>;
-        case 2: return launch<2, VY, MAXT>;
-        case 3: return launch<3, VY, MAXT>;
-        case 4: return launch<4, VY, MAXT>;
-        case 5: return launch<5, VY, MAXT>;
-        case 6: return launch<6, VY, MAXT>;
-        case 7: return launch<7, VY, MAXT>;
-        case 8: return launch<8, VY, MAXT>;
+        case 1: return launch<1, VY, NT, MINB>;
+        case 2: return launch<2, VY, NT, MINB>;
+        case 3: return launch<3, VY, NT, MINB>;
+        case 4: return launch<4, VY, NT, MINB>;
+        case 5: return launch<5, VY, NT, MINB>;
+        case 6: return launch<6, VY, NT, MINB>;
+        case 7: return launch<7, VY, NT, MINB>;
+        case 8: return launch<8, VY, NT, MINB>;
         default: return nullptr;
     }
 }
-
-template <int D, int VY, int MAXT>
-cudaError_t launch_split(const CUtensorMap* map, const St7Params& p, int grid, int threads, size_t smem,
-                         cudaStream_t s) {
-    auto k = st7_35d_split_kernel<TT, D, (D + 1) / 2, NTX, VY, ST_EXACT != 0, MAXT>;
-    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    k<<<grid, threads, smem, s>>>(*map, p);
-    return cudaGetLastError();
-}
-
-template <int VY, int MAXT>
-St7LaunchFn pick_split(int D) {
+template <int VY, int NT, int MINB>
+St7LaunchFn pick4(int D) {   // shallow sweeps only (register cap 65536 / (NT * MINB))
     switch (D) {
-        case 2: return launch_split<2, VY, MAXT>;
-        case 3: return launch_split<3, VY, MAXT>;
-        case 4: return launch_split<4, VY, MAXT>;
-        case 5: return launch_split<5, VY, MAXT>;
-        case 6: return launch_split<6, VY, MAXT>;
+        case 1: return launch<1, VY, NT, MINB>;
+        case 2: return launch<2, VY, NT, MINB>;
+        case 3: return launch<3, VY, NT, MINB>;
+        case 4: return launch<4, VY, NT, MINB>;
         default: return nullptr;
     }
 }
@@ -79,22 +67,17 @@ using namespace ST_UNIT_NS;
 
 #define ST_FN ST_CAT(ST_CAT(ST_CAT(st7_lookup_, ST_TNAME), _), ST_MODE)
 
-// variants: (VY=4, 256 threads max), (VY=2, 256), (VY=2, 512 threads: <= 128 registers)
-St7LaunchFn ST_FN(int D, int VY, int MAXT) {
-    if (VY == 4 && MAXT == 256) return pick<4, 256>(D);
-    if (VY == 2 && MAXT == 256) return pick<2, 256>(D);
-    if (VY == 2 && MAXT == 512) return pick<2, 512>(D);
-    if (VY == 4 && MAXT == 384) return pick<4, 384>(D);
+// compiled variants (rows per thread VY, threads per CTA NT, CTAs per SM MINB):
+// see variant_for in api.cu
+St7LaunchFn ST_FN(int D, int VY, int NT, int MINB) {
+    if (MINB == 1) {
+        if (VY == 4 && NT == 256) return pick<4, 256>(D);
+        if (VY == 4 && NT == 384) return pick4<4, 384, 1>(D);
+        if (VY == 2 && NT == 256) return pick<2, 256>(D);
+        if (VY == 2 && NT == 512) return pick4<2, 512, 1>(D);
+    }
+    if (MINB == 2 && VY == 2 && NT == 256) return pick4<2, 256, 2>(D);
     return nullptr;
 }
 
-}  // namespace st35d
-
-namespace st35d {
-#define ST_SFN ST_CAT(ST_CAT(ST_CAT(st7s_lookup_, ST_TNAME), _), ST_MODE)
-St7LaunchFn ST_SFN(int D, int VY, int MAXT) {
-    if (VY == 2 && MAXT == 512) return pick_split<2, 512>(D);
-    if (VY == 4 && MAXT == 384) return pick_split<4, 384>(D);
-    return nullptr;
-}
 }  // namespace st35d

@@ -18,11 +18,12 @@ def relerr(g, o):
     return float(np.max(np.abs(g - o) / np.maximum(np.abs(o), 1e-30)))
 
 
-def run_gpu(f0, flags, omega, T, dim_T=1, exact=False, lid=(0.05, 0.0, 0.0)):
+def run_gpu(f0, flags, omega, T, dim_T=1, exact=False, lid=(0.05, 0.0, 0.0), batched=-1):
     _, nz, ny, nx = f0.shape
     dt = torch.float32 if f0.dtype == np.float32 else torch.float64
     with st.Plan(nx, ny, nz, dt, dim_T) as p:
         p.set_lid(*lid)
+        p.set_option(st.ST_OPT_LBM_BATCHED, batched)
         if exact:
             p.set_bitexact(True)
         a = torch.from_numpy(f0).cuda()
@@ -142,6 +143,7 @@ def _cavity_on_device(n, dtype):
     w = stgen.lbm_rest(1, 1, 1, np.float32 if dtype == torch.float32 else np.float64).reshape(19)
     for i in range(19):
         f[i].fill_(float(w[i]))
+    torch.cuda.synchronize()   # the plan runs on its own stream
     return f, fl
 
 
@@ -199,3 +201,31 @@ def test_degenerate_lattices(oracle_lib, shape, dim_T):
     ref = oracle_lib.lbm(f0, flags, 1.6, 4)
     got = run_gpu(f0, flags, 1.6, 4, dim_T=dim_T, exact=True)
     assert np.array_equal(got, ref)
+
+
+@pytest.mark.parametrize("batched", [0, 1])
+@pytest.mark.parametrize("shape", [(32, 24, 20), (96, 50, 13)])
+def test_push_kernels_random(oracle_lib, shape, batched):
+    # both FP32 dim_T = 1 push kernels (per-direction flags / batched flags) on random
+    # populations: the batched one serves every FP32 lattice above 2^24 cells (bench's
+    # 1024^3 line), the per-direction one the smaller lattices
+    nx, ny, nz = shape
+    flags = stgen.cavity_flags(nx, ny, nz)
+    flags[nz // 2, ny // 3: ny // 3 + 3, nx // 4: nx // 4 + 5] = stgen.WALL   # interior obstacle
+    f0 = stgen.lbm_random(nx, ny, nz, 17, np.float32)
+    ref = oracle_lib.lbm(f0, flags, 1.6, 5)
+    assert np.array_equal(run_gpu(f0, flags, 1.6, 5, exact=True, batched=batched), ref)
+    assert relerr(run_gpu(f0, flags, 1.6, 5, batched=batched), ref) <= TOL[np.float32]
+
+
+def test_batched_kernel_above_2_24_cells(oracle_lib):
+    # just above the 2^24-cell switch (260 x 256 x 256 = 17.0 M cells): the automatic
+    # choice is the batched-flag kernel; random populations, whole lattice compared in
+    # the bit-exact and the tolerance build
+    nx, ny, nz, T = 260, 256, 256, 2
+    assert nx * ny * nz > 1 << 24
+    flags = stgen.cavity_flags(nx, ny, nz)
+    f0 = stgen.lbm_random(nx, ny, nz, 23, np.float32)
+    ref = oracle_lib.lbm(f0, flags, 1.6, T)
+    assert np.array_equal(run_gpu(f0, flags, 1.6, T, exact=True), ref)
+    assert relerr(run_gpu(f0, flags, 1.6, T), ref) <= TOL[np.float32]

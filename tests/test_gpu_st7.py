@@ -45,7 +45,7 @@ def test_config1_64cube(oracle_lib, dtype):
     assert np.array_equal(got, ref)
 
 
-SHAPES = [(68, 52, 37), (128, 96, 20), (16, 9, 5), (200, 70, 11)]
+SHAPES = [(68, 52, 37), (128, 96, 20), (16, 9, 5), (200, 70, 11), (64, 130, 9)]
 
 
 @pytest.mark.parametrize("dtype", [np.float32, np.float64])
@@ -60,7 +60,7 @@ def test_ragged_all_depths(oracle_lib, dtype, dim_T):
         got, _ = run_gpu(a, 0.4, 0.1, T, dim_T, exact=True)
         assert np.array_equal(got, ref), (nx, ny, nz, T)
         got, _ = run_gpu(a, 0.4, 0.1, T, dim_T)
-        assert relerr(got, ref) <= TOL[dtype] * max(1, T / 10), (nx, ny, nz, T)
+        assert relerr(got, ref) <= TOL[dtype], (nx, ny, nz, T)
 
 
 def test_dimT_invariance_bitexact():
@@ -106,8 +106,14 @@ def test_errors():
             p.st7(x, x, 0.4, 0.1, 3)                 # aliasing
         with pytest.raises(st.StError):
             p.st7(x, torch.empty_like(x), 0.4, 0.1, -1)
-        with pytest.raises(st.StError):
-            p.st7(x, np.empty((64, 64, 64), np.float32), 0.4, 0.1, 1)  # mixed host/device
+        with pytest.raises(ValueError):                 # mixed host/device (binding check)
+            p.st7(x, np.empty((64, 64, 64), np.float32), 0.4, 0.1, 1)
+        with pytest.raises(st.StError):                 # mixed host/device (C ABI check)
+            st.st7_run(p.h, x, np.empty((64, 64, 64), np.float32), 0.4, 0.1, 1)
+        with pytest.raises(ValueError):                 # short buffer
+            p.st7(x, torch.empty(64, 64, 63, device="cuda"), 0.4, 0.1, 1)
+        with pytest.raises(ValueError):                 # dtype does not match the plan
+            p.st7(x.double(), torch.empty(64, 64, 64, dtype=torch.float64, device="cuda"), 0.4, 0.1, 1)
 
 
 @pytest.mark.parametrize("dtype,dim_T", [(np.float32, 3), (np.float32, 4), (np.float64, 3)])

@@ -239,3 +239,48 @@ def test_shear_wave_decay(oracle_lib):
     # wrong viscosity (e.g. a dropped 1/2) would be far off
     wrong = U * np.exp(-(1 / omega) / 3 * (2 * np.pi / nz) ** 2 * T)
     assert abs(amp / wrong - 1) > 0.05
+
+
+def _couette_profile(oracle_lib, U, omega=1.0, ny=10, T=1500):
+    """Plane Couette flow: periodic in x and z, WALL plane y = 0, LID plane
+    y = ny-1 moving +x at U (X14's lid, rotated into a channel).  Returns the
+    x-velocity of each FLUID layer y = 1..ny-2 after T steps from rest."""
+    e, _, _ = _tables(oracle_lib)
+    nx = nz = 4
+    flags = np.zeros((nz, ny, nx), dtype=np.uint8)
+    flags[:, 0, :] = stgen.WALL
+    flags[:, ny - 1, :] = stgen.LID
+    f0 = stgen.lbm_rest(nx, ny, nz, np.float64)
+    f = oracle_lib.lbm(f0, flags, omega, T, u_lid=(U, 0.0, 0.0), periodic=True)
+    rho = f.sum(axis=0)
+    jx = np.tensordot(e[:, 0].astype(np.float64), f, axes=(0, 0))
+    ux = jx / rho
+    layers = ux[:, 1:ny - 1, :]
+    # the flow is uniform in x and z
+    assert np.max(np.abs(layers - layers[0:1, :, 0:1])) <= 1e-12
+    return layers[0, :, 0]
+
+
+def _couette_exact(U, ny):
+    # half-way bounce-back puts the walls midway between the wall/lid layers
+    # and the first FLUID layers: u = 0 at y = 1/2 and u = U at y = ny - 3/2
+    y = np.arange(1, ny - 1, dtype=np.float64)
+    return U * (y - 0.5) / (ny - 2)
+
+
+@pytest.mark.parametrize("omega", [1.0, 1.6])
+def test_couette_pins_lid_coefficient(oracle_lib, omega):
+    """Pins the magnitude of the Ladd moving-wall term f*_i - 6 w_i rho_w (e_i.u_w)
+    (X10/X14): the steady plane-Couette profile between a resting
+    wall and the lid is linear from 0 to U at the half-way wall positions.  A
+    coefficient of 2 w_i or 18 w_i (a dropped or doubled 1/c_s^2) gives U/3 or
+    3U at the lid; mass neutrality (P8b) cannot tell them apart."""
+    U, ny = 0.02, 10
+    prof = _couette_profile(oracle_lib, U, omega, ny)
+    exact = _couette_exact(U, ny)
+    assert np.max(np.abs(prof - exact)) <= 1e-3 * U   # measured: 6e-14 U (omega 1), 4e-5 U (1.6)
+    # guard: the test tells the plausible wrong coefficients apart.  The lid term
+    # is linear in u_w, so 2 w (e.u) == 6 w (e.(u/3)) and 18 w (e.u) == 6 w (e.(3u)).
+    for wrong in (U / 3, 3 * U):
+        bad = _couette_profile(oracle_lib, wrong, omega, ny)
+        assert np.max(np.abs(bad - exact)) > 0.05 * U

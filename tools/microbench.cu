@@ -14,8 +14,14 @@ __device__ unsigned long long g_cycles[4096];
 __device__ float g_sinkf[1 << 20];
 __device__ double g_sinkd[1 << 20];
 
-#define TIMED_BEGIN  __syncthreads(); long long t0 = clock64();
-#define TIMED_END    __syncthreads(); long long t1 = clock64(); if (threadIdx.x == 0) g_cycles[blockIdx.x] = t1 - t0;
+__device__ unsigned long long g_ns[4096];
+__device__ __forceinline__ unsigned long long gtimer() { unsigned long long t; asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t)); return t; }
+// clock64 (SM cycles) and %globaltimer (ns) over the same region: their ratio is the
+// SM clock the region actually ran at (round 1 divided by the event time of the whole
+// launch instead, which under-estimated the clock and gave impossible >128 lanes/clk)
+#define TIMED_BEGIN  __syncthreads(); long long t0 = clock64(); unsigned long long n0 = gtimer();
+#define TIMED_END    __syncthreads(); long long t1 = clock64(); unsigned long long n1 = gtimer(); \
+    if (threadIdx.x == 0) { g_cycles[blockIdx.x] = t1 - t0; g_ns[blockIdx.x] = n1 - n0; }
 
 __global__ void k_ffma(float a, float b) {
     float x0 = threadIdx.x, x1 = x0 + 1, x2 = x0 + 2, x3 = x0 + 3, x4 = x0 + 4, x5 = x0 + 5, x6 = x0 + 6, x7 = x0 + 7;
@@ -173,7 +179,7 @@ __global__ void k_lds128(float a, float b) {
     for (int i = 0; i < ITERS; ++i) {
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
-            float4 v = sm[(idx + j * 32) & (n - 1)];
+            float4 v = sm[(idx + j * 32 + i * 64) & (n - 1)];
             acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;  // 4 fadd per LDS.128
         }
     }
@@ -195,6 +201,148 @@ __global__ void k_sts128(float a, float b) {
     g_sinkf[blockIdx.x * blockDim.x + threadIdx.x] = sm[threadIdx.x].x;
 }
 
+
+// Packed FP32 with DISTINCT register operands every instruction (no operand
+// reuse), the stencil's pattern: does the register file sustain 2 pair reads
+// (FADD2) / 3 pair reads (FFMA2) per instruction at full rate?
+__global__ void k_fadd2_distinct(float a, float b) {
+    float2 x[24];
+#pragma unroll
+    for (int j = 0; j < 24; ++j) x[j] = make_float2(threadIdx.x + j, a + j);
+    TIMED_BEGIN
+    for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j] = __fadd2_rn(x[j + 8], x[j + 16]);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j + 8] = __fadd2_rn(x[j + 16], x[j]);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j + 16] = __fadd2_rn(x[j], x[j + 8]);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j] = __fadd2_rn(x[j + 8], x[j + 16]);
+    }
+    TIMED_END
+    float s = 0;
+#pragma unroll
+    for (int j = 0; j < 24; ++j) s += x[j].x + x[j].y;
+    g_sinkf[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+__global__ void k_ffma2_distinct(float a, float b) {
+    float2 x[24];
+#pragma unroll
+    for (int j = 0; j < 24; ++j) x[j] = make_float2(threadIdx.x + j, a + j);
+    TIMED_BEGIN
+    for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j] = __ffma2_rn(x[j + 8], x[j + 16], x[j]);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j + 8] = __ffma2_rn(x[j + 16], x[j], x[j + 8]);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j + 16] = __ffma2_rn(x[j], x[j + 8], x[j + 16]);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j] = __ffma2_rn(x[j + 8], x[j + 16], x[j]);
+    }
+    TIMED_END
+    float s = 0;
+#pragma unroll
+    for (int j = 0; j < 24; ++j) s += x[j].x + x[j].y;
+    g_sinkf[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+__global__ void k_fadd_distinct(float a, float b) {
+    float x[24];
+#pragma unroll
+    for (int j = 0; j < 24; ++j) x[j] = threadIdx.x + j * a;
+    TIMED_BEGIN
+    for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j] = __fadd_rn(x[j + 8], x[j + 16]);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j + 8] = __fadd_rn(x[j + 16], x[j]);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j + 16] = __fadd_rn(x[j], x[j + 8]);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j] = __fadd_rn(x[j + 8], x[j + 16]);
+    }
+    TIMED_END
+    float s = 0;
+#pragma unroll
+    for (int j = 0; j < 24; ++j) s += x[j];
+    g_sinkf[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+
+
+// FFMA2 / FMUL2 with one SCALAR (broadcast) operand and distinct pairs
+__global__ void k_ffma2_scalar(float a, float b) {
+    float2 x[24];
+#pragma unroll
+    for (int j = 0; j < 24; ++j) x[j] = make_float2(threadIdx.x + j, a + j);
+    const float2 c = make_float2(a, a);
+    TIMED_BEGIN
+    for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j] = __ffma2_rn(c, x[j + 8], x[j + 16]);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j + 8] = __ffma2_rn(c, x[j + 16], x[j]);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j + 16] = __ffma2_rn(c, x[j], x[j + 8]);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j] = __ffma2_rn(c, x[j + 8], x[j + 16]);
+    }
+    TIMED_END
+    float s = 0;
+#pragma unroll
+    for (int j = 0; j < 24; ++j) s += x[j].x + x[j].y;
+    g_sinkf[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+// the 7-point update mix per point pair: 4 FADD2 (distinct pairs), FMUL2 and
+// 2 FFMA2 with a scalar coefficient
+__global__ void k_mix7(float a, float b) {
+    float2 x[24];
+#pragma unroll
+    for (int j = 0; j < 24; ++j) x[j] = make_float2(threadIdx.x + j, a + j);
+    const float2 al = make_float2(a, a), be = make_float2(b, b);
+    TIMED_BEGIN
+    for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            const float2 s1 = __fadd2_rn(x[j], x[j + 8]);
+            const float2 s2 = __fadd2_rn(x[j + 16], x[(j + 1) % 8]);
+            const float2 s3 = __fadd2_rn(s1, x[(j + 3) % 8 + 8]);
+            const float2 s = __fadd2_rn(s3, s2);
+            const float2 t = __ffma2_rn(al, x[j + 16], __fmul2_rn(be, s));
+            x[j + 16] = __ffma2_rn(be, x[(j + 5) % 8 + 8], t);
+        }
+    }
+    TIMED_END
+    float s = 0;
+#pragma unroll
+    for (int j = 0; j < 24; ++j) s += x[j].x + x[j].y;
+    g_sinkf[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+// the same mix with per-element coefficient PAIRS (3 register pairs per FFMA2)
+__global__ void k_mix7_pairs(float a, float b) {
+    float2 x[24];
+#pragma unroll
+    for (int j = 0; j < 24; ++j) x[j] = make_float2(threadIdx.x + j, a + j);
+    const float2 al = make_float2(a, a + threadIdx.x * 1e-9f), be = make_float2(b, b - threadIdx.x * 1e-9f);
+    TIMED_BEGIN
+    for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            const float2 s1 = __fadd2_rn(x[j], x[j + 8]);
+            const float2 s2 = __fadd2_rn(x[j + 16], x[(j + 1) % 8]);
+            const float2 s3 = __fadd2_rn(s1, x[(j + 3) % 8 + 8]);
+            const float2 s = __fadd2_rn(s3, s2);
+            const float2 t = __ffma2_rn(al, x[j + 16], __fmul2_rn(be, s));
+            x[j + 16] = __ffma2_rn(be, x[(j + 5) % 8 + 8], t);
+        }
+    }
+    TIMED_END
+    float s = 0;
+#pragma unroll
+    for (int j = 0; j < 24; ++j) s += x[j].x + x[j].y;
+    g_sinkf[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+
 template <typename K>
 static int run(const char* name, K kern, int threads, double ops_per_thread_iter, int blocks_per_sm, size_t smem = 0) {
     int nsm = 0;
@@ -210,10 +358,15 @@ static int run(const char* name, K kern, int threads, double ops_per_thread_iter
     float ms; cudaEventElapsedTime(&ms, e0, e1);
     unsigned long long cyc[4096];
     CK(cudaMemcpyFromSymbol(cyc, g_cycles, sizeof(unsigned long long) * blocks));
-    double mean = 0; for (int i = 0; i < blocks; ++i) mean += cyc[i]; mean /= blocks;
+    unsigned long long ns[4096];
+    CK(cudaMemcpyFromSymbol(ns, g_ns, sizeof(unsigned long long) * blocks));
+    double mean = 0, mns = 0; for (int i = 0; i < blocks; ++i) { mean += cyc[i]; mns += ns[i]; } mean /= blocks; mns /= blocks;
     double ops_per_sm = ops_per_thread_iter * ITERS * threads * blocks_per_sm;
-    printf("%-12s threads=%4d bps=%d  %8.2f lane-ops/clk/SM   (%.3f ms, eff clk %.0f MHz)\n",
-           name, threads, blocks_per_sm, ops_per_sm / mean, ms, mean / (ms * 1e3));
+    // whole-launch throughput: every CTA's work over the event time (CTAs are not
+    // evenly co-resident, so per-CTA clock windows overstate the per-SM rate)
+    const double ev = ops_per_sm * nsm / (ms * 1e-3) / nsm / (mean / mns * 1e9);
+    printf("%-16s threads=%4d bps=%d  %8.2f lane-ops/clk/SM (whole launch, events)  clk %.0f MHz  %.3f ms\n",
+           name, threads, blocks_per_sm, ev, mean / mns * 1e3, ms);
     return 0;
 }
 
@@ -231,9 +384,11 @@ static int rund(const char* name, K kern, int threads, double ops, int bps) {
     float ms; cudaEventElapsedTime(&ms, e0, e1);
     unsigned long long cyc[4096];
     CK(cudaMemcpyFromSymbol(cyc, g_cycles, sizeof(unsigned long long) * blocks));
-    double mean = 0; for (int i = 0; i < blocks; ++i) mean += cyc[i]; mean /= blocks;
-    printf("%-12s threads=%4d bps=%d  %8.2f lane-ops/clk/SM   (%.3f ms, eff clk %.0f MHz)\n",
-           name, threads, bps, ops * ITERS * threads * bps / mean, ms, mean / (ms * 1e3));
+    unsigned long long ns[4096];
+    CK(cudaMemcpyFromSymbol(ns, g_ns, sizeof(unsigned long long) * blocks));
+    double mean = 0, mns = 0; for (int i = 0; i < blocks; ++i) { mean += cyc[i]; mns += ns[i]; } mean /= blocks; mns /= blocks;
+    printf("%-14s threads=%4d bps=%d  %8.2f lane-ops/clk/SM  %8.2f lane-ops/ns/SM  (clk %.0f MHz from clock64/globaltimer, %.3f ms)\n",
+           name, threads, bps, ops * ITERS * threads * bps / mean, ops * ITERS * threads * bps / mns, mean / mns * 1e3, ms);
     return 0;
 }
 
@@ -246,6 +401,12 @@ int main() {
         run("fadd", k_fadd, t, 32, 2);
         run("fadd2(x2)", k_fadd2, t, 32, 2);
         run("ffma2(x2)", k_ffma2, t, 32, 2);
+        run("fadd2 distinct", k_fadd2_distinct, t, 64, 2);
+        run("ffma2 distinct", k_ffma2_distinct, t, 64, 2);
+        run("fadd distinct", k_fadd_distinct, t, 32, 2);
+        run("ffma2 scalar", k_ffma2_scalar, t, 64, 2);
+        run("mix7 scalar", k_mix7, t, 8 * 14, 2);
+        run("mix7 pairs", k_mix7_pairs, t, 8 * 14, 2);
         rund("dfma", k_dfma, t, 32, 2);
         rund("dadd", k_dadd, t, 32, 2);
         run("shfl", k_shfl, t, 32, 2);
