@@ -46,6 +46,10 @@ def lib():
             fn.argtypes = [P, P, ctypes.c_long, ctypes.c_long, ctypes.c_long] + [ctypes.c_double] * 4 + \
                 [ctypes.c_int]
             fn.restype = ctypes.c_int
+            fn = getattr(L, f"oracle_st13_{sfx}")
+            fn.argtypes = [P, P, ctypes.c_long, ctypes.c_long, ctypes.c_long] + [ctypes.c_double] * 3 + \
+                [ctypes.c_int]
+            fn.restype = ctypes.c_int
             fn = getattr(L, f"oracle_lbm_{sfx}")
             fn.argtypes = [P, P, P, ctypes.c_long, ctypes.c_long, ctypes.c_long,
                            ctypes.c_double, ctypes.c_int, ctypes.c_double, ctypes.c_double,
@@ -91,6 +95,19 @@ def st27(A0: np.ndarray, alpha: float, beta: float, gamma: float, delta: float, 
         A0.ctypes.data, out.ctypes.data, nx, ny, nz, alpha, beta, gamma, delta, T)
     if rc != 0:
         raise RuntimeError(f"oracle_st27 rc={rc}")
+    return out
+
+
+def st13(A0: np.ndarray, alpha: float, beta: float, gamma: float, T: int) -> np.ndarray:
+    """T Jacobi sweeps of the radius-2 13-point star (general R of §V; X25),
+    Dirichlet shell 2 points thick (X26)."""
+    A0 = np.ascontiguousarray(A0)
+    nz, ny, nx = A0.shape
+    out = np.empty_like(A0)
+    rc = getattr(lib(), f"oracle_st13_{_sfx(A0.dtype)}")(
+        A0.ctypes.data, out.ctypes.data, nx, ny, nz, alpha, beta, gamma, T)
+    if rc != 0:
+        raise RuntimeError(f"oracle_st13 rc={rc}")
     return out
 
 

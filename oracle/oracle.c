@@ -12,7 +12,9 @@
  * 3.5D blocking only reorders the computation ("performing dim_T time steps
  * only requires grid elements to be read and written once"), so the
  * oracle is the plain definition: T naive Jacobi sweeps of
- *   - the 7-point stencil, P:111 (eq. in §IV-A1), and
+ *   - the 7-point stencil, P:111 (eq. in §IV-A1),
+ *   - the radius-2 13-point star (general R of §V; readings X25/X26),
+ *   - the 27-point stencil, and
  *   - the D3Q19 lattice-Boltzmann step, P:125-132 (§IV-B, push form).
  * Readings of silent/ambiguous points are DESIGN.md X1..X21.
  *
@@ -77,6 +79,61 @@ int oracle_st7_##SUFFIX(const TYPE* A0, TYPE* out, long nx, long ny, long nz,   
 }
 DEFINE_ST7(float, f32)
 DEFINE_ST7(double, f64)
+
+/* ------------------------------------------------------------------------ */
+/* Radius-2 star stencil, 13 points (the paper's general   */
+/* radius R of §V, "the radius (in units) of extent of the stencil,    */
+/* usually defined as the Manhattan distance (e.g. k-point stencil)", used   */
+/* in every blocking formula of §V, but only run with R = 1,      */
+/* P:259).  Reading X25 (the paper gives no R = 2 kernel):                    */
+/*   B = (alpha*C + beta*S1) + gamma*S2                                      */
+/*   S1 = ((x-1 + x+1) + (y-1 + y+1)) + (z-1 + z+1)   (the 7-point order X2) */
+/*   S2 = ((x-2 + x+2) + (y-2 + y+2)) + (z-2 + z+2)                          */
+/* three separately rounded products, 10 + 2 additions.  Reading X26: the    */
+/* fixed (Dirichlet) shell is R = 2 points thick on every face (the points   */
+/* whose stencil would leave the grid never change, as z0 in P:195).         */
+/* With alpha = 1 - 7.5 nu, beta = 4 nu / 3, gamma = -nu / 12 this is the    */
+/* explicit heat step with the 4th-order Laplacian (exact on polynomials of  */
+/* degree <= 5, the pin of tests/test_oracle_st13.py).                       */
+/* ------------------------------------------------------------------------ */
+#define DEFINE_ST13(TYPE, SUFFIX)                                                     \
+int oracle_st13_##SUFFIX(const TYPE* A0, TYPE* out, long nx, long ny, long nz,        \
+                         double alpha_d, double beta_d, double gamma_d, int T)        \
+{                                                                                     \
+    if (nx < 1 || ny < 1 || nz < 1 || T < 0) return -1;                               \
+    const size_t n = (size_t)nx * ny * nz;                                            \
+    const TYPE alpha = (TYPE)alpha_d, beta = (TYPE)beta_d, gamma = (TYPE)gamma_d;     \
+    TYPE* a = (TYPE*)malloc(n * sizeof(TYPE));                                        \
+    TYPE* b = (TYPE*)malloc(n * sizeof(TYPE));                                        \
+    if (!a || !b) { free(a); free(b); return -2; }                                    \
+    memcpy(a, A0, n * sizeof(TYPE));                                                  \
+    memcpy(b, A0, n * sizeof(TYPE));          /* both grids carry the shell */        \
+    for (int t = 0; t < T; ++t) {                                                     \
+        _Pragma("omp parallel for schedule(static)")                                  \
+        for (long z = 2; z < nz - 2; ++z)                                             \
+            for (long y = 2; y < ny - 2; ++y)                                         \
+                for (long x = 2; x < nx - 2; ++x) {                                   \
+                    TYPE sx1 = a[IDX(x - 1, y, z)] + a[IDX(x + 1, y, z)];             \
+                    TYPE sy1 = a[IDX(x, y - 1, z)] + a[IDX(x, y + 1, z)];             \
+                    TYPE sz1 = a[IDX(x, y, z - 1)] + a[IDX(x, y, z + 1)];             \
+                    TYPE sx2 = a[IDX(x - 2, y, z)] + a[IDX(x + 2, y, z)];             \
+                    TYPE sy2 = a[IDX(x, y - 2, z)] + a[IDX(x, y + 2, z)];             \
+                    TYPE sz2 = a[IDX(x, y, z - 2)] + a[IDX(x, y, z + 2)];             \
+                    TYPE s1 = (sx1 + sy1) + sz1;                                      \
+                    TYPE s2 = (sx2 + sy2) + sz2;                                      \
+                    TYPE p = alpha * a[IDX(x, y, z)];                                 \
+                    TYPE q = beta * s1;                                               \
+                    TYPE r = gamma * s2;                                              \
+                    b[IDX(x, y, z)] = (p + q) + r;                                    \
+                }                                                                     \
+        TYPE* tmp = a; a = b; b = tmp;           /* swap roles */              \
+    }                                                                                 \
+    memcpy(out, a, n * sizeof(TYPE));                                                 \
+    free(a); free(b);                                                                 \
+    return 0;                                                                         \
+}
+DEFINE_ST13(float, f32)
+DEFINE_ST13(double, f64)
 
 /* ------------------------------------------------------------------------ */
 /* 27-point stencil: the 3x3x3 cube around the      */
