@@ -103,6 +103,21 @@ int st7_run(st_plan* plan, const void* in, void* out, double alpha, double beta,
 int st27_run(st_plan* plan, const void* in, void* out, double alpha, double beta, double gamma, double delta, int T);
 
 /*
+ * st13_run — out = A(T): T Jacobi sweeps of the radius-2 13-point star, the
+ * general stencil radius R of §V ("the radius ... usually defined as
+ * the Manhattan distance (e.g. k-point stencil)") with R = 2 (SURVEY §8(f)
+ * f4; the paper runs only R = 1).  Reading X25:
+ *     B = (alpha*C + beta*S1) + gamma*S2
+ *     S1 = ((x-1 + x+1) + (y-1 + y+1)) + (z-1 + z+1), S2 likewise at distance 2
+ * Reading X26: the fixed (Dirichlet) shell is 2 points thick on every face.
+ * Sweeps of depth min(dim_T, 4 FP32 / 3 FP64) are kept on chip (3.5D, halo 2*dim_T,
+ * lag R per level).  Requires every extent >= 5.  Same buffers, ownership
+ * (`in` is scratch), pointer kinds and errors as st7_run; single process only.
+ * Bit-identical to the oracle with st_plan_set_bitexact(plan, 1).
+ */
+int st13_run(st_plan* plan, const void* in, void* out, double alpha, double beta, double gamma, int T);
+
+/*
  * lbm_d3q19_run — f_dst = state after T D3Q19 steps of f_src,
  * BGK single-relaxation collision with relaxation rate omega (0 <= omega < 2;
  * omega = 0 is pure streaming), push semantics: the stored state is

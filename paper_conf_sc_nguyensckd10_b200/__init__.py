@@ -46,7 +46,7 @@ class st_blocking(ctypes.Structure):
 
 _lib = None
 
-EXPORTS = ["st_plan_create", "st7_run", "st27_run", "lbm_d3q19_run", "st_destroy", "st_last_error", "st_last_status",
+EXPORTS = ["st_plan_create", "st7_run", "st13_run", "st27_run", "lbm_d3q19_run", "st_destroy", "st_last_error", "st_last_status",
            "st_plan_set_stream", "st_plan_set_option", "st_plan_set_lbm_lid", "st_plan_set_bitexact", "st_plan_set_variant", "st_plan_autotune", "st_plan_sync",
            "st_plan_set_dist", "st_plan_set_loopback_slabs", "st_plan_ghost_planes", "st_plan_local_slab",
            "st_plan_get_info", "st_plan_last_launches", "st_blocking_model", "st_fig3_step",
@@ -66,6 +66,7 @@ def lib() -> ctypes.CDLL:
         "st_plan_create": ([I, I, I, I, I], P),
         "st7_run": ([P, P, P, D, D, I], I),
         "st27_run": ([P, P, P, D, D, D, D, I], I),
+        "st13_run": ([P, P, P, D, D, D, I], I),
         "lbm_d3q19_run": ([P, P, P, D, I, P], I),
         "st_destroy": ([P], None),
         "st_last_error": ([], ctypes.c_char_p),
@@ -134,6 +135,10 @@ def st_plan_create(nx: int, ny: int, nz: int, dtype: int, dim_T: int) -> int:
 
 def st7_run(plan: int, inp, out, alpha: float, beta: float, T: int) -> int:
     return _check(lib().st7_run(plan, _ptr(inp), _ptr(out), alpha, beta, T))
+
+
+def st13_run(plan: int, inp, out, alpha: float, beta: float, gamma: float, T: int) -> int:
+    return _check(lib().st13_run(plan, _ptr(inp), _ptr(out), alpha, beta, gamma, T))
 
 
 def st27_run(plan: int, inp, out, alpha: float, beta: float, gamma: float, delta: float, T: int) -> int:
@@ -312,6 +317,10 @@ class Plan:
     def st7(self, inp, out, alpha: float, beta: float, T: int) -> None:
         self._check_bufs((inp, out), 1, "st7")
         st7_run(self.h, inp, out, alpha, beta, T)
+
+    def st13(self, inp, out, alpha: float, beta: float, gamma: float, T: int) -> None:
+        self._check_bufs((inp, out), 1, "st13")
+        st13_run(self.h, inp, out, alpha, beta, gamma, T)
 
     def st27(self, inp, out, alpha: float, beta: float, gamma: float, delta: float, T: int) -> None:
         self._check_bufs((inp, out), 1, "st27")

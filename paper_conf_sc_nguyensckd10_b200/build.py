@@ -49,6 +49,7 @@ UNITS = [
     ("lbm_inst.cu", "lbm_inst.o", []),
     ("naive.cu", "naive.o", []),
     ("st27.cu", "st27.o", []),
+    ("st13_inst.cu", "st13_inst.o", []),
     ("model.cpp", "model.o", []),
 ] + [
     ("st7_inst.cu", f"st7_{tn}_{mode}.o", [f"-DST_T={t}", f"-DST_TNAME={tn}", f"-DST_EXACT={ex}"])

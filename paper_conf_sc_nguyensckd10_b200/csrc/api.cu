@@ -13,6 +13,7 @@
 #include "../../include/st35d.h"
 #include "launch.h"
 #include "dist.h"
+#include "st13_kernel.cuh"
 
 using namespace st35d;
 
@@ -86,6 +87,7 @@ struct Geo7 {
     size_t smem = 0;
     double kappa = 0;
     St7LaunchFn fn = nullptr;
+    St13LaunchFn fn13 = nullptr;             // radius-2 plans
 };
 
 struct st_plan {
@@ -169,13 +171,15 @@ static size_t smem7(const Geo7& g, st_dtype dt, int ring) {
 // block, the last tile is placed so that y = ny-1 is the first row of a block;
 // no halo is needed beyond a grid face (the shell is fixed), so the first and
 // last tiles write up to the face
-static void place_y(Geo7& g, int ny, int d) {
-    g.wy = g.TY - 2 * d;
-    g.ey = ((g.VY - 1 - d) % g.VY + g.VY) % g.VY;
+// (R = stencil radius: the shell is R rows thick and the halo R*d rows)
+static void place_y(Geo7& g, int ny, int d, int R = 1) {
+    const int h = R * d;
+    g.wy = g.TY - 2 * h;
+    g.ey = ((g.VY - R - h) % g.VY + g.VY) % g.VY;   // y = R-1 on the last row of a block
     g.ly_last = g.oy0_last = 0;
-    if (g.TY - d - g.ey >= ny) { g.tiles_y = 1; return; }
-    g.ly_last = ny - 1 - (g.TY - g.VY);
-    g.oy0_last = std::max(g.ly_last + d, 0);
+    if (g.TY - h - g.ey >= ny) { g.tiles_y = 1; return; }
+    g.ly_last = ny - R - (g.TY - g.VY);              // y = ny-R on the first row of a block
+    g.oy0_last = std::max(g.ly_last + h, 0);
     g.tiles_y = std::max(1, (g.oy0_last + g.ey + g.wy - 1) / g.wy) + 1;
 }
 
@@ -233,6 +237,54 @@ static int get_geo7(st_plan* p, int d, int nzo, Geo7*& out) {
     // grid depends on the output-plane count of the call
     const long long work = (long long)out->tiles_x * out->tiles_y * nzo;
     out->grid = (int)std::min<long long>((long long)p->sms * out->minb, std::max<long long>(work, 1));
+    return ST_OK;
+}
+
+
+// ----------------------------------------------------------------------------
+// radius-2 (13-point star) planner: the 7-point planner with R = 2 (halo 2d,
+// shell 2 rows thick, ring keeps 3 planes, exchange 2 rows per side for 3 rounds)
+// ----------------------------------------------------------------------------
+static size_t smem13(const Geo7& g, st_dtype dt, int ring) {
+    return (size_t)ring * g.TX * g.TY * esize(dt) + (size_t)(g.d > 1 ? g.d - 1 : 0) * 3 * 4 * g.threads * 16 +
+           ST7_RING_MAX * 8;
+}
+
+static int plan13(st_plan* p, int d, int nzo, Geo7& g) {
+    const int R = 2;
+    g.d = d;
+    g.VX = p->dtype == ST_F32 ? 4 : 2;
+    g.NTX = p->dtype == ST_F32 ? 16 : 32;
+    g.TX = g.NTX * g.VX;
+    g.VY = d <= 2 ? 4 : 2;
+    g.maxt = 256;
+    g.minb = 1;
+    g.hx = (R * d + g.VX - 1) / g.VX * g.VX;
+    g.wx = (g.TX - g.hx - R * d) & ~(g.VX - 1);
+    if (g.wx < g.VX) return fail(ST_EUNSUPPORTED, "radius 2: dim_T %d too deep for the %d-wide tile", d, g.TX);
+    g.tiles_x = (p->nx + g.wx - 1) / g.wx;
+    long best = -1;
+    for (int nty = 2; nty <= g.maxt / g.NTX; ++nty) {
+        Geo7 c = g;
+        c.NTY = nty;
+        c.TY = nty * c.VY;
+        c.threads = c.NTX * nty;
+        if (c.TY - 2 * R * d < 1) continue;
+        place_y(c, p->ny, d, R);
+        c.ring = 0;
+        for (int r = ST7_RING_MAX; r >= 4; --r)
+            if (smem13(c, p->dtype, r) <= p->smem_optin) { c.ring = r; break; }
+        if (c.ring < 4) continue;
+        c.smem = smem13(c, p->dtype, c.ring);
+        const long cost = (long)c.tiles_y * c.TY;
+        if (best < 0 || cost < best || (cost == best && c.TY > g.TY)) { best = cost; g = c; }
+    }
+    if (best < 0) return fail(ST_EUNSUPPORTED, "radius 2: dim_T %d too deep for the tiles of this build", d);
+    const long long work = (long long)g.tiles_x * g.tiles_y * nzo;
+    g.grid = (int)std::min<long long>(p->sms, std::max<long long>(work, 1));
+    g.kappa = (double)g.tiles_x * g.TX * g.tiles_y * g.TY / ((double)p->nx * p->ny);
+    g.fn13 = st13_lookup(p->dtype == ST_F32 ? 0 : 1, p->exact, d, g.VY);
+    if (!g.fn13) return fail(ST_EUNSUPPORTED, "no radius-2 kernel for dim_T %d", d);
     return ST_OK;
 }
 
@@ -809,6 +861,83 @@ extern "C" int st27_run(st_plan* p, const void* in, void* out, double alpha, dou
     if (rc) return rc;
     CUDA_TRY(cudaMemcpyAsync(p->hbuf[0], in, n, cudaMemcpyHostToDevice, p->stream));
     rc = run27_device(p, p->hbuf[0], p->hbuf[1], w, T);
+    if (rc) return rc;
+    CUDA_TRY(cudaMemcpyAsync(out, p->hbuf[1], n, cudaMemcpyDeviceToHost, p->stream));
+    CUDA_TRY(cudaStreamSynchronize(p->stream));
+    return ST_OK;
+}
+
+// ----------------------------------------------------------------------------
+// Radius-2 13-point star (general R of §V; X25/X26):
+// ceil(T/D) ping-pong sweeps of st13_kernel.cuh, D = min(dim_T, 4 FP32 / 3 FP64); single
+// process only.
+// ----------------------------------------------------------------------------
+static int launch13(st_plan* p, const void* src, void* dst, int d, const double w[3]) {
+    Geo7 g;
+    int rc = plan13(p, d, p->nz, g);
+    if (rc) return rc;
+    CUtensorMap map;
+    rc = encode_3d(&map, src, p->dtype, p->nx, p->ny, p->nz, g.TX, g.TY);
+    if (rc) return rc;
+    St13Params prm{};
+    St7Params& q = prm.g;
+    q.out = dst;
+    q.nx = p->nx; q.ny = p->ny; q.nzb = p->nz; q.zbase = 0; q.nzg = p->nz;
+    q.za = 0; q.zb = p->nz;
+    q.tiles_x = g.tiles_x; q.ntiles = g.tiles_x * g.tiles_y;
+    q.wx = g.wx; q.wy = g.wy; q.hx = g.hx;
+    q.tiles_y = g.tiles_y; q.ey = g.ey; q.ly_last = g.ly_last; q.oy0_last = g.oy0_last;
+    q.ring = g.ring;
+    q.pdl = p->opt_pdl;
+    q.alpha = w[0]; q.beta = w[1]; prm.gamma = w[2];
+    if ((long long)q.ntiles * p->nz >= (1LL << 31)) return fail(ST_EUNSUPPORTED, "grid too large");
+    const int grid = std::min(g.grid, ST7_MAX_GRID);
+    split_work(q.ntiles, p->nz, 2 * d, grid, q.split);
+    cudaError_t e = g.fn13(&map, prm, grid, g.threads, g.smem, p->stream);
+    if (e != cudaSuccess) return fail(ST_ECUDA, "st13 launch (d=%d): %s", d, cudaGetErrorString(e));
+    ++p->launches;
+    return ST_OK;
+}
+
+static int run13_device(st_plan* p, const void* in, void* out, const double w[3], int T) {
+    const size_t n = (size_t)p->nx * p->ny * p->nz * esize(p->dtype);
+    p->launches = 0;
+    if (T == 0) {
+        CUDA_TRY(cudaMemcpyAsync(out, in, n, cudaMemcpyDeviceToDevice, p->stream));
+        return ST_OK;
+    }
+    // FP64 at depth 4 needs 16 halo rows per side: no 256-thread tile fits
+    const std::vector<int> ds = sweep_depths(T, std::min(p->dimT, p->dtype == ST_F32 ? ST13_MAX_DIM_T : 3));
+    void* bufs[2] = {const_cast<void*>(in), out};
+    for (size_t k = 0; k < ds.size(); ++k) {
+        int rc = launch13(p, bufs[k % 2], bufs[(k + 1) % 2], ds[k], w);
+        if (rc) return rc;
+    }
+    if (ds.size() % 2 == 0) CUDA_TRY(cudaMemcpyAsync(out, in, n, cudaMemcpyDeviceToDevice, p->stream));
+    CUDA_TRY(cudaGetLastError());
+    return ST_OK;
+}
+
+extern "C" int st13_run(st_plan* p, const void* in, void* out, double alpha, double beta, double gamma, int T) {
+    if (!p) return fail(ST_EINVAL, "NULL plan");
+    if (!in || !out) return fail(ST_EINVAL, "NULL grid pointer");
+    if (T < 0) return fail(ST_EINVAL, "T = %d < 0", T);
+    if (p->dist.mode != Dist::SINGLE) return fail(ST_EUNSUPPORTED, "st13_run is single-process only");
+    if (p->nx < 5 || p->ny < 5 || p->nz < 5) return fail(ST_EINVAL, "radius 2 needs every extent >= 5");
+    const size_t n = (size_t)p->nx * p->ny * p->nz * esize(p->dtype);
+    if (overlap(in, out, n)) return fail(ST_EINVAL, "in and out overlap");
+    const int kin = ptr_kind(in), kout = ptr_kind(out);
+    if (kin != kout) return fail(ST_EINVAL, "in and out must both be host or both be device pointers");
+    const double w[3] = {alpha, beta, gamma};
+    if (kin == 1) {
+        if ((reinterpret_cast<uintptr_t>(in) | reinterpret_cast<uintptr_t>(out)) & 15)
+            return fail(ST_EINVAL, "device grids must be 16-byte aligned");
+        return run13_device(p, in, out, w, T);
+    }
+    int rc = ensure_hbuf(p, n);
+    if (rc) return rc;
+    CUDA_TRY(cudaMemcpyAsync(p->hbuf[0], in, n, cudaMemcpyHostToDevice, p->stream));
+    rc = run13_device(p, p->hbuf[0], p->hbuf[1], w, T);
     if (rc) return rc;
     CUDA_TRY(cudaMemcpyAsync(out, p->hbuf[1], n, cudaMemcpyDeviceToHost, p->stream));
     CUDA_TRY(cudaStreamSynchronize(p->stream));

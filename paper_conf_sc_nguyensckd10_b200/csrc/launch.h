@@ -37,6 +37,13 @@ St7LaunchFn st7_lookup_f32_exact(int D, int VY, int NT, int MINB);
 St7LaunchFn st7_lookup_f64_fast(int D, int VY, int NT, int MINB);
 St7LaunchFn st7_lookup_f64_exact(int D, int VY, int NT, int MINB);
 
+// radius-2 (13-point star) sweep (st13_kernel.cuh); nullptr if (D, VY) is not compiled
+struct St13Params;
+using St13LaunchFn = cudaError_t (*)(const CUtensorMap* map, const St13Params& p, int grid, int threads, size_t smem,
+                                     cudaStream_t s);
+St13LaunchFn st13_lookup(int dtype, bool exact, int D, int VY);
+constexpr int ST13_MAX_DIM_T = 4;
+
 bool lbm_push_batched(int esize, int nx, int ny, int nzb, int force);   // kernel choice (also sets the grid)
 cudaError_t lbm_push_launch(int dtype, bool exact, bool slab, bool batched, const void* src, void* dst,
                             const uint8_t* fl2, const LbmParams& p, int grid, cudaStream_t s);

@@ -32,6 +32,10 @@
 
 namespace st35d {
 
+#ifndef ST27_STEP3
+#define ST27_STEP3 0
+#endif
+
 namespace {
 template <typename T, bool EX> struct Op;
 template <> struct Op<float, true> {
@@ -105,6 +109,15 @@ __global__ void __launch_bounds__(NTHR, MINB) st27_kernel(const T* __restrict__ 
 
     // Z windows: level L (0..D-1) as a source, slot k holds (a, f, e) of one plane
     T wa[D][3][VY], wf[D][3][VY], we[D][3][VY];
+    // zero-initialised: the first rounds of a chunk read window slots that no
+    // earlier round has written (their results are never stored, but reading
+    // an indeterminate value is undefined behaviour the compiler may exploit)
+#pragma unroll
+    for (int L = 0; L < D; ++L)
+#pragma unroll
+        for (int k = 0; k < 3; ++k)
+#pragma unroll
+            for (int j = 0; j < VY; ++j) wa[L][k][j] = wf[L][k][j] = we[L][k][j] = T(0);
     // level-0 planes arrive PF-1 rounds ahead through a per-thread cp.async
     // ring (each thread copies and later reads only its own VY elements, so no
     // barrier guards the ring; the loads stay in flight across the rounds'
@@ -202,6 +215,19 @@ __global__ void __launch_bounds__(NTHR, MINB) st27_kernel(const T* __restrict__ 
     const bool tile_shell = x0 == 0 || x0 + TW >= p.nx || y0 == 0 || y0 + TH >= p.ny;
     using S1 = std::true_type;
     using S0 = std::false_type;
+#if ST27_STEP3
+    // A/B: the three rotation bodies in sequence from a loop stepping by three
+    for (int i = 0; i < nround; i += 3) {
+        const bool sh0 = tile_shell || lo0 + i - D <= 0 || lo0 + i - 1 >= p.nz - 1;
+        if (sh0) round(i, std::integral_constant<int, 0>{}, S1{}); else round(i, std::integral_constant<int, 0>{}, S0{});
+        if (i + 1 >= nround) break;
+        const bool sh1 = tile_shell || lo0 + i + 1 - D <= 0 || lo0 + i >= p.nz - 1;
+        if (sh1) round(i + 1, std::integral_constant<int, 1>{}, S1{}); else round(i + 1, std::integral_constant<int, 1>{}, S0{});
+        if (i + 2 >= nround) break;
+        const bool sh2 = tile_shell || lo0 + i + 2 - D <= 0 || lo0 + i + 1 >= p.nz - 1;
+        if (sh2) round(i + 2, std::integral_constant<int, 2>{}, S1{}); else round(i + 2, std::integral_constant<int, 2>{}, S0{});
+    }
+#else
     for (int i = 0; i < nround; ++i) {
         const int r = i % 3;
         const bool sh = tile_shell || lo0 + i - D <= 0 || lo0 + i - 1 >= p.nz - 1;
@@ -215,6 +241,9 @@ __global__ void __launch_bounds__(NTHR, MINB) st27_kernel(const T* __restrict__ 
             else round(i, std::integral_constant<int, 2>{}, S0{});
         }
     }
+#endif
+    // the last rounds re-copy the chunk's last plane into the ring: drain them
+    asm volatile("cp.async.wait_all;" ::: "memory");
 }
 
 template <typename T, int D, bool EX>
