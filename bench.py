@@ -39,6 +39,11 @@ SM_COUNT = 148
 FP32_LANES, FP64_LANES = 128, 64
 ST7_OPS = 7            # FP instructions per 7-point update: 5 add, 1 mul, 1 fma (8 flops)
 ST27_OPS = 16          # FP instructions per 27-point update in the plane-factorised order X24: 12 add + 4 mul
+ST13_OPS = 13          # FP lane-ops per radius-2 update (X25 with FMA): 9 add, 1 mul, 3 fma
+# measured FP32 throughput of the 7-point instruction mix (4 FADD2, FMUL2, 2 FFMA2 with a
+# scalar coefficient, distinct register pairs): tools/microbench.cu "mix7 scalar", 512
+# threads x 2 CTAs per SM, profiles/r02/microbench.txt -- above the 128-lane nominal
+MIX7_LANE_OPS_PER_CLK_SM = 167.7
 LBM_BYTES = {4: 153, 8: 305}   # (19*2*E + 1) per LBM update at dim_T = 1 (X12)
 
 
@@ -115,6 +120,14 @@ class ClockSampler:
         s = sorted(self.samples)
         return {"sm_mhz": s[len(s) // 2] if s else None, "sm_max_mhz": self.max_mhz,
                 "reasons": sorted(self.reasons), "samples": len(s)}
+
+
+def n_sweeps(T, D):
+    """sweeps of a T-step run at depth D: ceil(T/D), made odd (the library's sweep_depths)"""
+    S = (T + D - 1) // D
+    if S % 2 == 0 and S < T:
+        S += 1
+    return S
 
 
 def load_traffic(key):
@@ -309,22 +322,34 @@ def main():
         per_launch_ms = ms / launches
         d_eff = info["dim_t_sweep"]
         upd_rank = upd / world
-        # roofline of the dominant kernel (st7_35d): both roofs, report the binding one
-        ops_peak = SM_COUNT * FP32_LANES * sm_max * 1e6 / 1e12          # T FP32 lane-ops/s
+        # roofline of the dominant kernel (st7_35d, the only kernel of the step): both roofs,
+        # the binding one first.  Algorithmic bytes: every sweep reads and writes the grid
+        # once (2 E n^3 per sweep); the sweep count (incl. the remainder sweeps that
+        # make it odd) comes from the run itself (launches per step).
+        ops_peak = SM_COUNT * FP32_LANES * sm_max * 1e6 / 1e12          # T FP32 lane-ops/s (nominal lanes)
+        ops_peak_mix = SM_COUNT * MIX7_LANE_OPS_PER_CLK_SM * sm_max * 1e6 / 1e12
         achieved_ops = ST7_OPS * upd_rank / (ms / 1e3) / 1e12
-        bytes_per_upd = 8.0 / D
-        achieved_gbs = bytes_per_upd * upd_rank / (ms / 1e3) / 1e9
+        sweeps = n_sweeps(T, d_eff)
+        bytes_step = 2 * 4 * n * n * n * sweeps                  # per rank (its n^3 slab)
+        bytes_per_upd = bytes_step / upd_rank
+        achieved_gbs = bytes_step / (ms / 1e3) / 1e9
         hbm_roof_upd = hbm_gbs * 1e9 / bytes_per_upd
         alu_roof_upd = ops_peak * 1e12 / ST7_OPS
         traffic = load_traffic(f"st7_f32_{n}_D{D}")
         r_alu = {"bound": "alu", "achieved": round(achieved_ops, 3), "peak": round(ops_peak, 2),
-                 "unit": "Top/s (FP32 lane-instructions; 7 per update)",
+                 "unit": "Top/s (FP32 lane-ops; 7 per update)",
                  "frac": round(achieved_ops / ops_peak, 4), "traffic": traffic,
-                 "peak_source": f"148 SM x 128 FP32 lanes x {sm_max:.0f} MHz (clocks.max.sm)"}
+                 "frac_of_measured_mix": round(achieved_ops / ops_peak_mix, 4),
+                 "peak_source": f"148 SM x 128 FP32 lanes x {sm_max:.0f} MHz (clocks.max.sm); "
+                                f"frac_of_measured_mix uses the microbenchmarked 7-point mix, "
+                                f"{MIX7_LANE_OPS_PER_CLK_SM} lane-ops/clk/SM"}
         r_hbm = {"bound": "hbm", "achieved": round(achieved_gbs, 1), "peak": hbm_gbs, "unit": "GB/s",
                  "frac": round(achieved_gbs / hbm_gbs, 4), "traffic": traffic,
-                 "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_src}); algorithmic 8/dim_T B/update"}
+                 "bytes_per_update": round(bytes_per_upd, 4),
+                 "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_src}); algorithmic 2E n^3 per sweep, "
+                                f"{sweeps} sweeps per step"}
         roof, alt = (r_hbm, r_alu) if hbm_roof_upd < alu_roof_upd else (r_alu, r_hbm)
+        roof = dict(roof, frac_hbm=r_hbm["frac"], frac_fp=r_alu["frac"])
 
     # ------------------------------------------------------------------ e2e (host buffers)
     a_host = torch.from_numpy(host0).pin_memory()
@@ -380,30 +405,78 @@ def main():
                 "note": f"{ST27_OPS} FP instructions per update (plane-factorised order X24, no FMA); "
                         "the paper's definition counts 30 (4 mul + 26 add, P:119)"}
             del x27, y27
-        # ablation ladder (Fig. 5(b)): no blocking -> 2.5D (dim_T = 1)
-        # -> 3.5D (measured dim_T), same grid and T; plus the eq. (3) model's dim_T seed (f3)
+        # radius-2 13-point star on the configs[1] grid, T = 100, every depth
+        for dtn, dt_np, tdt, dmax, lanes in (("f32", np.float32, torch.float32, 4, 128),
+                                             ("f64", np.float64, torch.float64, 3, FP64_LANES)):
+            x13 = torch.from_numpy(stgen.grid7(n, n, n, 2, dt_np)).cuda()
+            y13 = torch.empty_like(x13)
+            sw13 = {}
+            w13 = (1 - 7.5 * 0.05, 4 * 0.05 / 3, -0.05 / 12)
+            for d in range(1, dmax + 1):
+                with st.Plan(n, n, n, tdt, d) as p13:
+                    p13.set_stream(stream)
+                    t13, _ = time_steps(lambda: p13.st13(x13, y13, *w13, T), 2, 1)
+                    sw13[d] = round((n - 4) ** 3 * T / (t13 / 2 / 1e3) / 1e6, 1)
+            d13 = max(sw13, key=sw13.get)
+            v13 = sw13[d13] * 1e6
+            E13 = 4 if dtn == "f32" else 8
+            b13 = 2 * E13 * n ** 3 * n_sweeps(T, d13) / ((n - 4) ** 3 * T)
+            extras[f"st13_{dtn}_256"] = {
+                "value": sw13[d13], "unit": "Mupdates/s", "dim_T": d13, "dim_T_sweep": sw13,
+                "roofline_hbm": {"achieved": round(b13 * v13 / 1e9, 1), "peak": hbm_gbs, "unit": "GB/s",
+                                 "frac": round(b13 * v13 / 1e9 / hbm_gbs, 4)},
+                "frac_alu": round(ST13_OPS * v13 / (SM_COUNT * lanes * sm_max * 1e6), 4),
+                "note": f"radius 2, interior (n-4)^3 points; {ST13_OPS} FP lane-ops per update (X25 with FMA)"}
+            del x13, y13
+        # ablation ladder (Fig. 5(b)), FP32 256^3, T = 100:
+        # no blocking -> 2.5D spatial (dim_T = 1) -> 4D (3D blocks of 64 planes + temporal,
+        # P:349) -> 3.5D with one row of points per thread -> + several rows per thread
+        # (multi-update) -> + two-phase rounds (ILP, the production kernel)
         xa = torch.from_numpy(stgen.grid7(n, n, n, 2, np.float32)).cuda()
         ya = torch.empty_like(xa)
-        with st.Plan(n, n, n, torch.float32, 1) as pn:
-            pn.set_stream(stream)
-            pn.set_variant(st.ST_VARIANT_NAIVE)
-            tn, _ = time_steps(lambda: pn.st7(xa, ya, 0.4, 0.1, T), 2, 1)
-        with st.Plan(n, n, n, torch.float32, 8) as pa:   # the library's own depth selection (f3)
+
+        def bar(D_, variant=0, zchunk=0, naive=False):
+            with st.Plan(n, n, n, torch.float32, D_) as pb:
+                pb.set_stream(stream)
+                if naive:
+                    pb.set_variant(st.ST_VARIANT_NAIVE)
+                pb.set_option(st.ST_OPT_ST7_VARIANT, variant)
+                pb.set_option(st.ST_OPT_ZCHUNK, zchunk)
+                tb, _ = time_steps(lambda: pb.st7(xa, ya, 0.4, 0.1, T), 2, 1)
+                return round((n - 2) ** 3 * T / (tb / 2 / 1e3) / 1e6, 1)
+
+        def best_of(fn, depths=(2, 3, 4)):
+            r = {d: fn(d) for d in depths}
+            b = max(r, key=r.get)
+            return {"value": r[b], "dim_T": b, "dim_T_sweep": r}
+
+        ladder = {
+            "naive_no_blocking": {"value": bar(1, naive=True)},
+            "2.5D_spatial_dim_T_1": {"value": sweep.get(1) or bar(1)},
+            "4D_3D_blocks_64_planes": best_of(lambda d: bar(d, zchunk=64)),
+            "3.5D_one_row_per_thread": best_of(lambda d: bar(d, variant=1256)),
+            "3.5D_multi_update_level_by_level": best_of(lambda d: bar(d, variant=94256)),
+            "3.5D_multi_update_two_phase": {"value": round(value, 1), "dim_T": D},
+        }
+        with st.Plan(n, n, n, torch.float32, 8) as pa:   # the library's model-seeded depth search (f3)
             pa.set_stream(stream)
-            at_d, at_eta, at_ms = pa.autotune(xa, ya, 24)
+            rep = pa.autotune_report(xa, ya, 24)
         del xa, ya
         gamma = 8.0 / ST7_OPS                                    # B per FP instruction
-        Gamma = hbm_gbs * 1e9 / (ops_peak * 1e12)                # B200: measured HBM / FP32 lane-instr rate
+        Gamma = hbm_gbs * 1e9 / (ops_peak * 1e12)                # measured HBM / nominal FP32 lane rate
         mdl = st.st_blocking_model(227 * 1024, 4, 1, gamma, Gamma, 0, 0)
         extras["ablation_f32_256"] = {
-            "unit": "Mupdates/s", "naive_no_blocking": round((n - 2) ** 3 * T / (tn / 2 / 1e3) / 1e6, 1),
-            "2.5D_dim_T_1": sweep.get(1), "3.5D": round(value, 1), "dim_T": D,
-            "model": {"gamma_B_per_instr": round(gamma, 3), "Gamma_B_per_instr": round(Gamma, 4),
-                      "eta_eq3": mdl["eta"], "measured_best_dim_T": D,
-                      "st_plan_autotune": {"dim_T": at_d, "eta_seed_nominal_peaks": at_eta, "T_probe": 24,
-                                           "ms": {k: round(v, 4) for k, v in at_ms.items()}},
-                      "note": "eta = ceil(gamma/Gamma) is where the HBM roof meets the FP32 roof; the "
-                              "measured optimum is lower because the kernel is issue/latency-bound"}}
+            "unit": "Mupdates/s", "bars": ladder,
+            "note": "each bar's kernel is captured by tools/ladder_ncu.sh (profiles/r02/ladder/)"}
+        extras["model_f3"] = {
+            "gamma_B_per_op": round(gamma, 4), "Gamma_nominal_B_per_op": round(Gamma, 4), "eta_nominal": mdl["eta"],
+            "autotune": {k: (round(v, 6) if isinstance(v, float) else v) for k, v in rep.items()},
+            "predicted_dim_T": rep["eta"], "measured_best_dim_T": D, "autotune_choice": rep["dim_T"],
+            "tile_side_eq4": {"cta_smem": rep["tile_side"][0], "sm_smem_rf": rep["tile_side"][1],
+                              "cluster8_dsmem": rep["tile_side"][2]},
+            "tile_used": [info["tile_x"], info["tile_y"]],
+            "note": "eta = ceil(gamma/Gamma_eff) with Gamma_eff = measured depth-1 bytes/s over the deepest "
+                    "sweep's FP lane-ops/s; the nominal-peak eta assumes an FP-pipe-bound kernel"}
         # LBM D3Q19 cavity 256^3 (configs[2])
         for dtn, dt_np, tdt in (("f32", np.float32, torch.float32), ("f64", np.float64, torch.float64)):
             nl, Tl = 256, 100

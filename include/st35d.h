@@ -173,24 +173,62 @@ int st_plan_set_variant(st_plan* plan, int variant);
  *                       interior sweep on a side stream; 0 serialised.
  *   ST_OPT_PDL          1 (default): 7-point sweeps chained with programmatic
  *                       dependent launch; 0 plain launches.
- *   ST_OPT_ST7_VARIANT  0 (default) auto; else VY*1000 + threads per CTA of a
- *                       compiled 7-point kernel variant (4256, 4384, 2256).
+ *   ST_OPT_ST7_VARIANT  0 (default) auto; else VY*1000 + threads per CTA
+ *                       (+ 10000 * CTAs per SM) of a compiled 7-point kernel
+ *                       variant: 4256, 4384, 2256, 2512, 22256; FP32 ablation
+ *                       ladder: 1256 (one row per thread), 94256 (level by
+ *                       level, no two-phase rounds).
+ *   ST_OPT_ZCHUNK       0 (default); > 0: the 7-point sweep also restarts every
+ *                       that many output planes of a tile, i.e. 3D blocks with
+ *                       temporal blocking (the ablation ladder's 4D bar,
+ *                       PAPER.md P:275-281).
  * Results do not depend on any option.  Unknown option or value: ST_EINVAL. */
-enum { ST_OPT_LBM_BATCHED = 1, ST_OPT_LBM_KERNEL = 2, ST_OPT_OVERLAP = 3, ST_OPT_PDL = 4, ST_OPT_ST7_VARIANT = 5 };
+enum { ST_OPT_LBM_BATCHED = 1, ST_OPT_LBM_KERNEL = 2, ST_OPT_OVERLAP = 3, ST_OPT_PDL = 4, ST_OPT_ST7_VARIANT = 5,
+       ST_OPT_ZCHUNK = 6 };
 int st_plan_set_option(st_plan* plan, int option, int value);
 
-/* st_plan_autotune — choose the 7-point sweep depth by measurement (the
- * paper's "framework that determines the various blocking parameters", P:377,
- * eqs. (1)-(4) of §V-C).  Every depth 1..(deepest the plan tiles, <= dim_T)
- * runs T_probe Jacobi steps of st7_run on the caller's DEVICE grids a and b
- * (n^3 each, both clobbered), timed with CUDA events on the plan stream; the
- * fastest depth becomes the plan's st7_run sweep depth (results are identical
- * for every depth).  eta_out (may be NULL) receives the eq. (3) seed
- * eta = ceil(gamma/Gamma) with gamma = 2E/7 bytes per FP instruction and Gamma
- * = this device's nominal HBM bytes/s over its FP32 (FP64) lane-instr/s;
- * ms_out (may be NULL, length >= dim_T) receives the time per depth.
- * Synchronous.  Single-process plans only (ST_EUNSUPPORTED otherwise: tune
- * one rank and broadcast).  Returns the chosen depth (>= 1) or < 0. */
+/* st_plan_autotune_report — choose the 7-point sweep depth (the paper's
+ * "framework that determines the various blocking parameters"; eqs.
+ * (1)-(4) of §V-C) from a model seeded by measurement:
+ *   gamma     = 2E/7 bytes per FP lane-op of the 7-point update;
+ *   Gamma_eff = (bytes/s of a depth-1 sweep) / (FP lane-ops/s of the deepest
+ *               sweep the plan tiles): what this device delivers to this
+ *               kernel, issue limits included (the nominal-peak Gamma of
+ *               eq. (3) is reported beside it);
+ *   eta       = the smallest depth with dim_T / kappa(dim_T) >= gamma / Gamma_eff
+ *               (eq. 3 with the planner's overestimation kappa, eq. 2)
+ *               seeds the search: depths
+ *               eta-1..eta+1 are timed and the search walks toward the faster
+ *               neighbour until the best has timed neighbours on both sides;
+ *   tile_side = eq. (4) at eta for three on-chip capacities C: one CTA's
+ *               shared memory, the SM's shared memory + register file, and an
+ *               8-CTA cluster's distributed shared memory.
+ * Each timed depth runs T_probe Jacobi steps of st7_run on the caller's DEVICE
+ * grids a and b (n^3 each, both clobbered), CUDA events on the plan stream;
+ * results are identical for every depth.  The fastest depth becomes the
+ * plan's st7_run sweep depth.  Synchronous.  Single-process plans only
+ * (ST_EUNSUPPORTED otherwise: tune one rank and broadcast).  Returns the
+ * chosen depth (>= 1) or < 0; rep (may be NULL) receives the report. */
+typedef struct {
+    int dim_T;                 /* chosen depth                                      */
+    int eta;                   /* P:255 / eq. (3) with Gamma_eff and kappa          */
+    int eta_nominal;           /* eq. (3) with the device's nominal peaks           */
+    double gamma;              /* bytes per FP lane-op of the kernel                */
+    double Gamma_nominal;      /* nominal HBM bytes/s / FP lane-ops/s               */
+    double Gamma_eff;          /* measured (see above)                              */
+    double bw_dim1;            /* measured algorithmic bytes/s at depth 1           */
+    double fp_deep;            /* measured FP lane-ops/s at the deepest depth (ghost points incl.) */
+    int tested[ST_MAX_DIM_T];  /* 1 where the depth was timed                       */
+    float ms[ST_MAX_DIM_T];    /* time of T_probe steps per timed depth (0 untimed) */
+    double capacity[3];        /* C (bytes): CTA smem, SM smem + RF, 8-CTA cluster  */
+    int tile_side[3];          /* eq. (4) floor(sqrt(C / (E (2R+2) eta)))           */
+    double kappa[3];           /* eq. (2) at that side and eta                      */
+} st_autotune_report;
+int st_plan_autotune_report(st_plan* plan, void* a, void* b, int T_probe, st_autotune_report* rep);
+
+/* st_plan_autotune — the same search; eta_out (may be NULL) receives the
+ * eq. (3) eta from the measured Gamma, ms_out (may be NULL, length >=
+ * ST_MAX_DIM_T) the time per depth (0 for depths not timed). */
 int st_plan_autotune(st_plan* plan, void* a, void* b, int T_probe, int* eta_out, float* ms_out);
 
 /* Waits for the plan stream; returns ST_ECUDA for deferred device faults. */

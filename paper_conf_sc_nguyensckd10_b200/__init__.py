@@ -21,7 +21,7 @@ ST_F32, ST_F64 = 0, 1
 ST_OK, ST_EINVAL, ST_ENOMEM, ST_ECUDA, ST_ENCCL, ST_EUNSUPPORTED = 0, -1, -2, -3, -4, -5
 ST_FLUID, ST_WALL, ST_LID = 0, 1, 2
 ST_MAX_DIM_T = 8
-ST_OPT_LBM_BATCHED, ST_OPT_LBM_KERNEL, ST_OPT_OVERLAP, ST_OPT_PDL, ST_OPT_ST7_VARIANT = 1, 2, 3, 4, 5
+ST_OPT_LBM_BATCHED, ST_OPT_LBM_KERNEL, ST_OPT_OVERLAP, ST_OPT_PDL, ST_OPT_ST7_VARIANT, ST_OPT_ZCHUNK = 1, 2, 3, 4, 5, 6
 _ERRNAMES = {-1: "ST_EINVAL", -2: "ST_ENOMEM", -3: "ST_ECUDA", -4: "ST_ENCCL", -5: "ST_EUNSUPPORTED"}
 
 
@@ -39,6 +39,14 @@ class st_plan_info(ctypes.Structure):
                 ("ring", ctypes.c_int)]
 
 
+class st_autotune_report(ctypes.Structure):
+    _fields_ = [("dim_T", ctypes.c_int), ("eta", ctypes.c_int), ("eta_nominal", ctypes.c_int),
+                ("gamma", ctypes.c_double), ("Gamma_nominal", ctypes.c_double), ("Gamma_eff", ctypes.c_double),
+                ("bw_dim1", ctypes.c_double), ("fp_deep", ctypes.c_double),
+                ("tested", ctypes.c_int * ST_MAX_DIM_T), ("ms", ctypes.c_float * ST_MAX_DIM_T),
+                ("capacity", ctypes.c_double * 3), ("tile_side", ctypes.c_int * 3), ("kappa", ctypes.c_double * 3)]
+
+
 class st_blocking(ctypes.Structure):
     _fields_ = [("eta", ctypes.c_int), ("dim_bound", ctypes.c_double), ("dim", ctypes.c_int),
                 ("kappa", ctypes.c_double)]
@@ -47,7 +55,7 @@ class st_blocking(ctypes.Structure):
 _lib = None
 
 EXPORTS = ["st_plan_create", "st7_run", "st13_run", "st27_run", "lbm_d3q19_run", "st_destroy", "st_last_error", "st_last_status",
-           "st_plan_set_stream", "st_plan_set_option", "st_plan_set_lbm_lid", "st_plan_set_bitexact", "st_plan_set_variant", "st_plan_autotune", "st_plan_sync",
+           "st_plan_set_stream", "st_plan_set_option", "st_plan_set_lbm_lid", "st_plan_set_bitexact", "st_plan_set_variant", "st_plan_autotune", "st_plan_autotune_report", "st_plan_sync",
            "st_plan_set_dist", "st_plan_set_loopback_slabs", "st_plan_ghost_planes", "st_plan_local_slab",
            "st_plan_get_info", "st_plan_last_launches", "st_blocking_model", "st_fig3_step",
            "st_nccl_unique_id", "st_slab_range"]
@@ -77,6 +85,7 @@ def lib() -> ctypes.CDLL:
         "st_plan_set_bitexact": ([P, I], I),
         "st_plan_set_variant": ([P, I], I),
         "st_plan_autotune": ([P, P, P, I, ctypes.POINTER(I), ctypes.POINTER(ctypes.c_float)], I),
+        "st_plan_autotune_report": ([P, P, P, I, ctypes.POINTER(st_autotune_report)], I),
         "st_plan_sync": ([P], I),
         "st_plan_set_dist": ([P, P, I, I], I),
         "st_plan_set_loopback_slabs": ([P, I], I),
@@ -186,6 +195,17 @@ def st_plan_autotune(plan: int, a, b, T_probe: int):
     ms = (ctypes.c_float * 16)()
     d = _check(lib().st_plan_autotune(plan, _ptr(a), _ptr(b), T_probe, ctypes.byref(eta), ms))
     return d, eta.value, {k + 1: ms[k] for k in range(16) if ms[k] > 0}
+
+
+def st_plan_autotune_report(plan: int, a, b, T_probe: int) -> dict:
+    """model-seeded depth search (include/st35d.h); returns the report as a dict."""
+    r = st_autotune_report()
+    _check(lib().st_plan_autotune_report(plan, _ptr(a), _ptr(b), T_probe, ctypes.byref(r)))
+    out = {k: getattr(r, k) for k, _ in st_autotune_report._fields_}
+    for k in ("tested", "ms", "capacity", "tile_side", "kappa"):
+        out[k] = list(out[k])
+    out["ms"] = {d + 1: round(v, 4) for d, v in enumerate(out["ms"]) if v > 0}
+    return out
 
 
 def st_plan_sync(plan: int) -> int:
@@ -343,6 +363,9 @@ class Plan:
 
     def autotune(self, a, b, T_probe: int):
         return st_plan_autotune(self.h, a, b, T_probe)
+
+    def autotune_report(self, a, b, T_probe: int) -> dict:
+        return st_plan_autotune_report(self.h, a, b, T_probe)
 
     def set_variant(self, variant: int) -> None:
         st_plan_set_variant(self.h, variant)

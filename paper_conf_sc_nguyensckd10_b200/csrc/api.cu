@@ -110,7 +110,8 @@ struct st_plan {
     int opt_lbm_kernel = 0;     // 0 auto, 1 push, 2 multi-level
     int opt_overlap = 1;
     int opt_pdl = 1;
-    int opt_st7_variant = 0;    // 0 auto, else VY * 1000 + threads per CTA
+    int opt_st7_variant = 0;    // 0 auto, else VY * 1000 + threads per CTA (+ 10000 * CTAs per SM)
+    int opt_zchunk = 0;         // 0: z-runs as the work split gives; > 0: 3D blocks of that depth
     // host-pointer staging
     void* hbuf[2] = {nullptr, nullptr};
     size_t hbuf_bytes = 0;
@@ -154,6 +155,9 @@ static St7LaunchFn lookup7(st_dtype dt, bool exact, int d, int vy, int nt, int m
     if (dt == ST_F32) return exact ? st7_lookup_f32_exact(d, vy, nt, minb) : st7_lookup_f32_fast(d, vy, nt, minb);
     return exact ? st7_lookup_f64_exact(d, vy, nt, minb) : st7_lookup_f64_fast(d, vy, nt, minb);
 }
+
+// CTAs per SM of a variant (minb 9 = the ladder's level-by-level kernel, one per SM)
+static int ctas_per_sm(const Geo7& g) { return g.minb == 9 ? 1 : g.minb; }
 
 static size_t smem7(const Geo7& g, st_dtype dt, int ring) {
     // TMA ring + row exchange [D-1][2][2][threads] x 16 B + mbarriers + load cursor
@@ -208,7 +212,10 @@ static int plan7(st_plan* p, int d, int nzo, Geo7& g) {
         // ahead and must cover HBM latency, several rounds of compute)
         c.ring = 0;
         for (int r = ST7_RING_MAX; r >= 4; --r)
-            if (smem7(c, p->dtype, r) <= (g.minb == 1 ? p->smem_optin : p->smem_sm / g.minb - 1024)) { c.ring = r; break; }
+            if (smem7(c, p->dtype, r) <= (ctas_per_sm(g) == 1 ? p->smem_optin : p->smem_sm / ctas_per_sm(g) - 1024)) {
+                c.ring = r;
+                break;
+            }
         if (c.ring < 4) continue;
         c.smem = smem7(c, p->dtype, c.ring);
         const long cost = (long)c.tiles_y * c.TY;
@@ -216,7 +223,7 @@ static int plan7(st_plan* p, int d, int nzo, Geo7& g) {
     }
     if (best < 0) return fail(ST_EUNSUPPORTED, "dim_T %d too deep for the tiles of this build", d);
     const long long work = (long long)g.tiles_x * g.tiles_y * nzo;
-    g.grid = (int)std::min<long long>((long long)p->sms * g.minb, std::max<long long>(work, 1));
+    g.grid = (int)std::min<long long>((long long)p->sms * ctas_per_sm(g), std::max<long long>(work, 1));
     g.kappa = (double)g.tiles_x * g.TX * g.tiles_y * g.TY / ((double)p->nx * p->ny);
     g.fn = lookup7(p->dtype, p->exact, d, g.VY, ntmax, g.minb);
     if (!g.fn) return fail(ST_EUNSUPPORTED, "no kernel for dim_T %d (VY %d, %d threads)", d, g.VY, ntmax);
@@ -236,7 +243,7 @@ static int get_geo7(st_plan* p, int d, int nzo, Geo7*& out) {
     out = &it->second;
     // grid depends on the output-plane count of the call
     const long long work = (long long)out->tiles_x * out->tiles_y * nzo;
-    out->grid = (int)std::min<long long>((long long)p->sms * out->minb, std::max<long long>(work, 1));
+    out->grid = (int)std::min<long long>((long long)p->sms * ctas_per_sm(*out), std::max<long long>(work, 1));
     return ST_OK;
 }
 
@@ -378,6 +385,10 @@ extern "C" int st_plan_set_option(st_plan* p, int option, int value) {
             p->opt_lbm_kernel = value; return ST_OK;
         case ST_OPT_OVERLAP: p->opt_overlap = value != 0; return ST_OK;
         case ST_OPT_PDL: p->opt_pdl = value != 0; return ST_OK;
+        case ST_OPT_ZCHUNK:
+            if (value < 0) return fail(ST_EINVAL, "ST_OPT_ZCHUNK %d", value);
+            p->opt_zchunk = value;
+            return ST_OK;
         case ST_OPT_ST7_VARIANT:
             if (value != 0 && !lookup7(p->dtype, p->exact, 1, value / 1000 % 10, value % 1000, std::max(1, value / 10000)))
                 return fail(ST_EINVAL, "ST_OPT_ST7_VARIANT %d is not compiled", value);
@@ -485,7 +496,7 @@ static bool overlap(const void* a, const void* b, size_t n) {
 // levels, which run only some levels, plus the first plane's load latency;
 // calibrated by measurement below).  Minimises the largest cost by bisection
 // over a greedy cut.
-static void split_work(int ntiles, int nzo, int d, int G, int* split) {
+static void split_work(int ntiles, int nzo, int d, int G, int* split, int zchunk = 0) {
     const long long work = (long long)ntiles * nzo;
     // measured on B200 (ST_SPLIT_OVH A/B, 256^3): 4 plane-equivalents per segment is
     // best at dim_T 3 and 4 (+2 % over the d + 2 model); shallower sweeps restart cheaper
@@ -499,7 +510,8 @@ static void split_work(int ntiles, int nzo, int d, int G, int* split) {
             ++b;
             long long budget = C;
             while (it < work) {
-                const long long in_tile = (it / nzo + 1) * nzo - it;
+                long long in_tile = (it / nzo + 1) * nzo - it;
+                if (zchunk > 0) in_tile = std::min(in_tile, zchunk - (it % nzo) % zchunk);   // a 3D block
                 if (budget <= ovh) break;
                 const long long take = std::min(in_tile, budget - ovh);
                 it += take;
@@ -534,11 +546,12 @@ static int launch7(st_plan* p, const void* src, void* dst, int d, double alpha, 
     prm.tiles_y = g->tiles_y; prm.ey = g->ey; prm.ly_last = g->ly_last; prm.oy0_last = g->oy0_last;
     prm.ring = g->ring;
     prm.pdl = p->opt_pdl;
+    prm.zchunk = p->opt_zchunk;
     prm.alpha = alpha; prm.beta = beta;
     if ((long long)prm.ntiles * (sv.zb - sv.za) <= 0) return ST_OK;
     if ((long long)prm.ntiles * (sv.zb - sv.za) >= (1LL << 31)) return fail(ST_EUNSUPPORTED, "grid too large");
     const int grid = std::min(sv.grid_cap > 0 ? std::min(g->grid, sv.grid_cap) : g->grid, ST7_MAX_GRID);
-    split_work(prm.ntiles, sv.zb - sv.za, d, grid, prm.split);
+    split_work(prm.ntiles, sv.zb - sv.za, d, grid, prm.split, p->opt_zchunk);
     cudaError_t e = g->fn(&map, prm, grid, g->threads, g->smem, sv.stream ? sv.stream : p->stream);
     if (e != cudaSuccess) return fail(ST_ECUDA, "st7 launch (d=%d): %s", d, cudaGetErrorString(e));
     ++p->launches;
@@ -945,12 +958,31 @@ extern "C" int st13_run(st_plan* p, const void* in, void* out, double alpha, dou
 }
 
 // ----------------------------------------------------------------------------
-// Blocking-parameter selection by measurement ("a framework that
-// determines the various blocking parameters"): the eq. (3) bound eta from this
-// device's HBM bandwidth and FP issue rate seeds the report; every depth
-// 1..dimKmax is timed on the caller's grids and the fastest is kept.
+// Blocking-parameter selection ("a framework that determines the
+// various blocking parameters"; eqs. (1)-(4)): the eq. (3) bound
+// eta, the smallest depth with dim_T / kappa > gamma / Gamma (eq. (3)
+// with the overestimation kappa of the planner's tiling, eq. (2)), evaluated
+// with a Gamma MEASURED on this device and kernel -- the bytes/s of a depth-1
+// sweep (the bandwidth the kernel gets) over the FP lane-ops/s of the
+// deepest sweep (the rate its issue-limited compute reaches, ghost points
+// included) -- seeds the search; depths eta-1..eta+1 are timed and the
+// search walks on while a neighbour is faster, so the nominal-peak eta (6-7
+// on B200, where the kernel is not FP-pipe bound) never costs 8 timings.
 // ----------------------------------------------------------------------------
-extern "C" int st_plan_autotune(st_plan* p, void* a, void* b, int T_probe, int* eta_out, float* ms_out) {
+static int time_depth(st_plan* p, void* a, void* b, int d, int T_probe, cudaEvent_t e0, cudaEvent_t e1, float& ms) {
+    p->dimK = d;
+    int rc = run7_device(p, a, b, 0.4, 0.1, std::min(T_probe, 2 * d));   // warm-up (geometry, first launch)
+    if (rc) return rc;
+    cudaEventRecord(e0, p->stream);
+    rc = run7_device(p, a, b, 0.4, 0.1, T_probe);
+    if (rc) return rc;
+    cudaEventRecord(e1, p->stream);
+    if (cudaEventSynchronize(e1) != cudaSuccess) return fail(ST_ECUDA, "autotune: %s", cudaGetErrorString(cudaGetLastError()));
+    cudaEventElapsedTime(&ms, e0, e1);
+    return ST_OK;
+}
+
+extern "C" int st_plan_autotune_report(st_plan* p, void* a, void* b, int T_probe, st_autotune_report* rep) {
     if (!p) return fail(ST_EINVAL, "NULL plan");
     if (!a || !b) return fail(ST_EINVAL, "NULL grid pointer");
     if (T_probe < 1) return fail(ST_EINVAL, "T_probe = %d < 1", T_probe);
@@ -960,44 +992,107 @@ extern "C" int st_plan_autotune(st_plan* p, void* a, void* b, int T_probe, int* 
     if (ptr_kind(a) != 1 || ptr_kind(b) != 1) return fail(ST_EINVAL, "autotune needs device grids");
     if ((reinterpret_cast<uintptr_t>(a) | reinterpret_cast<uintptr_t>(b)) & 15)
         return fail(ST_EINVAL, "device grids must be 16-byte aligned");
-    if (eta_out) {   // eq. (3): gamma = 2E bytes / 7 FP instructions per update; Gamma of this device
+    st_autotune_report r;
+    memset(&r, 0, sizeof r);
+    const double E = (double)esize(p->dtype);
+    r.gamma = 2.0 * E / 7.0;                         // bytes per FP lane-op of the 7-point update
+    {   // nominal Gamma: device HBM bytes/s over FP lane-ops/s (FP32 128 / FP64 64 lanes per SM)
         int memclk_khz = 0, bus_bits = 0, smclk_khz = 0;
         cudaDeviceGetAttribute(&memclk_khz, cudaDevAttrMemoryClockRate, p->dev);
         cudaDeviceGetAttribute(&bus_bits, cudaDevAttrGlobalMemoryBusWidth, p->dev);
         cudaDeviceGetAttribute(&smclk_khz, cudaDevAttrClockRate, p->dev);
-        const double lanes = p->dtype == ST_F32 ? 128.0 : 64.0;   // FP32 / FP64 lanes per SM (sm_100)
+        const double lanes = p->dtype == ST_F32 ? 128.0 : 64.0;
         const double bw = 2.0 * memclk_khz * 1e3 * bus_bits / 8.0;
         const double ops = (double)p->sms * lanes * smclk_khz * 1e3;
+        r.Gamma_nominal = (bw > 0 && ops > 0) ? bw / ops : 0;
         st_blocking m{};
-        const double E = (double)esize(p->dtype);
-        *eta_out = (bw > 0 && ops > 0 && st_blocking_model(p->smem_optin, E, 1, 2.0 * E / 7.0, bw / ops, 0, 0, &m) == ST_OK)
-                       ? m.eta : 0;
+        r.eta_nominal = r.Gamma_nominal > 0 && st_blocking_model(p->smem_optin, E, 1, r.gamma, r.Gamma_nominal, 0, 0, &m) == ST_OK
+                            ? m.eta : 0;
     }
     cudaEvent_t e0, e1;
     CUDA_TRY(cudaEventCreate(&e0));
     CUDA_TRY(cudaEventCreate(&e1));
-    const int keep = p->dimK;
-    int best = keep;
-    float best_ms = 0.f;
+    const int keep = p->dimK, dmax = p->dimKmax;
+    const double upd = (double)(p->nx - 2) * (p->ny - 2) * (p->nz - 2) * T_probe;
     int rc = ST_OK;
-    for (int d = 1; d <= p->dimKmax && rc == ST_OK; ++d) {
-        p->dimK = d;
-        rc = run7_device(p, a, b, 0.4, 0.1, std::min(T_probe, 2 * d));   // warm-up (geometry, first launch)
-        if (rc) break;
-        cudaEventRecord(e0, p->stream);
-        rc = run7_device(p, a, b, 0.4, 0.1, T_probe);
-        if (rc) break;
-        cudaEventRecord(e1, p->stream);
-        if (cudaEventSynchronize(e1) != cudaSuccess) { rc = fail(ST_ECUDA, "autotune: %s", cudaGetErrorString(cudaGetLastError())); break; }
+    auto probe = [&](int d) -> float {
+        if (d < 1 || d > dmax) return 0.f;
+        if (r.ms[d - 1] > 0) return r.ms[d - 1];
         float ms = 0.f;
-        cudaEventElapsedTime(&ms, e0, e1);
-        if (ms_out) ms_out[d - 1] = ms;
-        if (d == 1 || ms < best_ms) { best = d; best_ms = ms; }
+        if (rc == ST_OK) rc = time_depth(p, a, b, d, T_probe, e0, e1, ms);
+        if (rc == ST_OK) { r.ms[d - 1] = ms; r.tested[d - 1] = 1; }
+        return rc == ST_OK ? ms : 0.f;
+    };
+    // measured Gamma: bytes/s at depth 1 (2E per point per sweep) over FP lane-ops/s at the deepest depth
+    const float m1 = probe(1), md = probe(dmax);
+    // kappa(d): loaded / useful points of the planner's tiling at depth d (eq. (2) analog)
+    auto kappa_at = [&](int d) {
+        Geo7* g = nullptr;
+        return get_geo7(p, d, p->dist.nzl, g) == ST_OK ? g->kappa : 1.0;
+    };
+    if (rc == ST_OK && m1 > 0 && md > 0) {
+        const double sweeps1 = (double)sweep_depths(T_probe, 1).size();
+        r.bw_dim1 = 2.0 * E * (double)p->nx * p->ny * p->nz * sweeps1 / (m1 * 1e-3);
+        // FP lane-ops the deepest sweep executes, redundant (ghost) points included
+        r.fp_deep = 7.0 * upd * kappa_at(dmax) / (md * 1e-3);
+        r.Gamma_eff = r.bw_dim1 / r.fp_deep;
+        // blocking pays while dim_T / kappa > gamma / Gamma -> the smallest such depth
+        r.eta = dmax;
+        for (int d = 1; d <= dmax; ++d)
+            if (d / kappa_at(d) >= r.gamma / r.Gamma_eff) { r.eta = d; break; }
+    }
+    // eq. (4) tile sides at eta for three on-chip capacities: one CTA's shared
+    // memory, the SM's shared memory + register file, an 8-CTA cluster's DSMEM
+    {
+        int regs = 0;
+        cudaDeviceGetAttribute(&regs, cudaDevAttrMaxRegistersPerMultiprocessor, p->dev);
+        const double caps[3] = {(double)p->smem_optin, (double)p->smem_sm + 4.0 * regs, 8.0 * p->smem_optin};
+        for (int c = 0; c < 3; ++c) {
+            st_blocking m{};
+            if (r.eta > 0 && st_blocking_model(caps[c], E, 1, r.gamma, r.gamma / r.eta, r.eta, 0, &m) == ST_OK) {
+                r.capacity[c] = caps[c];
+                r.tile_side[c] = m.dim;
+                r.kappa[c] = m.kappa;
+            }
+        }
+    }
+    // seed at eta, time its neighbours, walk toward the faster side
+    int best = 1;
+    if (rc == ST_OK) {
+        const int seed = std::max(1, std::min(r.eta > 0 ? r.eta : dmax, dmax));
+        for (int d = seed - 1; d <= seed + 1; ++d) probe(d);
+        auto best_tested = [&]() {
+            int b = 0;
+            for (int d = 1; d <= dmax; ++d)
+                if (r.ms[d - 1] > 0 && (b == 0 || r.ms[d - 1] < r.ms[b - 1])) b = d;
+            return b;
+        };
+        for (int guard = 0; guard < dmax && rc == ST_OK; ++guard) {
+            best = best_tested();
+            const int lo = best - 1, hi = best + 1;
+            const bool more = (lo >= 1 && r.ms[lo - 1] == 0) || (hi <= dmax && r.ms[hi - 1] == 0);
+            if (!more) break;
+            probe(lo);
+            probe(hi);
+        }
+        best = best_tested();
     }
     cudaEventDestroy(e0);
     cudaEventDestroy(e1);
     p->dimK = rc ? keep : best;
+    r.dim_T = rc ? 0 : best;
+    if (rep) *rep = r;
     return rc ? rc : best;
+}
+
+extern "C" int st_plan_autotune(st_plan* p, void* a, void* b, int T_probe, int* eta_out, float* ms_out) {
+    st_autotune_report r;
+    const int rc = st_plan_autotune_report(p, a, b, T_probe, &r);
+    if (rc < 0) return rc;
+    if (eta_out) *eta_out = r.eta;
+    if (ms_out)
+        for (int d = 0; d < ST_MAX_DIM_T; ++d) ms_out[d] = r.ms[d];
+    return rc;
 }
 
 // ----------------------------------------------------------------------------

@@ -28,9 +28,9 @@ namespace ST_UNIT_NS {
 using TT = ST_T;
 constexpr int NTX = sizeof(TT) == 4 ? 16 : 32;   // threads across the 64-point tile row
 
-template <int D, int VY, int NT, int MINB>
+template <int D, int VY, int NT, int MINB, bool SPLIT = true>
 cudaError_t launch(const CUtensorMap* map, const St7Params& p, int grid, int threads, size_t smem, cudaStream_t s) {
-    auto k = st7_35d_kernel<TT, D, NTX, VY, ST_EXACT != 0, NT, MINB>;
+    auto k = st7_35d_kernel<TT, D, NTX, VY, ST_EXACT != 0, NT, MINB, SPLIT>;
     if (threads > NT || threads % NTX) return cudaErrorInvalidValue;
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
@@ -51,13 +51,13 @@ St7LaunchFn pick(int D) {
         default: return nullptr;
     }
 }
-template <int VY, int NT, int MINB>
+template <int VY, int NT, int MINB, bool SPLIT = true>
 St7LaunchFn pick4(int D) {   // shallow sweeps only (register cap 65536 / (NT * MINB))
     switch (D) {
-        case 1: return launch<1, VY, NT, MINB>;
-        case 2: return launch<2, VY, NT, MINB>;
-        case 3: return launch<3, VY, NT, MINB>;
-        case 4: return launch<4, VY, NT, MINB>;
+        case 1: return launch<1, VY, NT, MINB, SPLIT>;
+        case 2: return launch<2, VY, NT, MINB, SPLIT>;
+        case 3: return launch<3, VY, NT, MINB, SPLIT>;
+        case 4: return launch<4, VY, NT, MINB, SPLIT>;
         default: return nullptr;
     }
 }
@@ -67,9 +67,14 @@ using namespace ST_UNIT_NS;
 
 #define ST_FN ST_CAT(ST_CAT(ST_CAT(st7_lookup_, ST_TNAME), _), ST_MODE)
 
-// compiled variants (rows per thread VY, threads per CTA NT, CTAs per SM MINB):
-// see variant_for in api.cu
+// compiled variants (rows per thread VY, threads per CTA NT, CTAs per SM MINB;
+// MINB = 9: the level-by-level round order of the ablation ladder): see
+// variant_for in api.cu
 St7LaunchFn ST_FN(int D, int VY, int NT, int MINB) {
+#if !ST_EXACT
+    if (sizeof(TT) == 4 && MINB == 9 && VY == 4 && NT == 256) return pick4<4, 256, 1, false>(D);   // ladder: no phase split
+    if (sizeof(TT) == 4 && MINB == 1 && VY == 1 && NT == 256) return pick4<1, 256, 1>(D);           // ladder: one row per thread
+#endif
     if (MINB == 1) {
         if (VY == 4 && NT == 256) return pick<4, 256>(D);
         if (VY == 4 && NT == 384) return pick4<4, 384, 1>(D);

@@ -39,10 +39,6 @@
 #include <type_traits>
 #include "common.cuh"
 
-#ifndef ST7_SPLIT
-#define ST7_SPLIT 1
-#endif
-
 namespace st35d {
 
 constexpr int ST7_MAX_GRID = 320;   // >= CTAs of one sweep (148 SMs x up to 2 CTAs per SM)
@@ -65,6 +61,8 @@ struct St7Params {
     // ly_last puts y = ny-1 on the first row, so y-shell rows never share a
     // thread with interior rows (their threads copy: coefficients (1, 0)).
     int tiles_y, ey, ly_last, oy0_last;
+    int zchunk;        // > 0: segments also end at multiples of zchunk output planes of a
+                       // tile (3D blocks: the ablation ladder's 4D bar); 0: z-runs as split
     int ring;          // TMA ring slots (<= ST7_RING_MAX); ring - 2 planes are prefetched ahead
     int pdl;           // host side: launch with programmatic dependent launch
     double alpha, beta;
@@ -260,8 +258,10 @@ __device__ __forceinline__ St7Tile st7_tile(const St7Params& p, int tile, int D)
     return t;
 }
 
-// NT threads per CTA, MINB CTAs per SM (register cap 65536 / (NT * MINB))
-template <typename T, int D, int NTX, int VY, bool EXACT, int NT, int MINB>
+// NT threads per CTA, MINB CTAs per SM (register cap 65536 / (NT * MINB));
+// SPLIT: two-phase rounds (false: level by level, the ablation ladder's
+// pre-ILP bar)
+template <typename T, int D, int NTX, int VY, bool EXACT, int NT, int MINB, bool SPLIT = true>
 __global__ void __launch_bounds__(NT, MINB)
 st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
     constexpr int VX = sizeof(T) == 4 ? 4 : 2;
@@ -332,7 +332,8 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
     auto seg_at = [&](int it) {
         Seg g;
         g.tile = it / nzo;
-        const int seg_end = min(item_end, (g.tile + 1) * nzo);
+        int seg_end = min(item_end, (g.tile + 1) * nzo);
+        if (p.zchunk > 0) seg_end = min(seg_end, it + (p.zchunk - (it - g.tile * nzo) % p.zchunk));
         g.za = p.za + (it - g.tile * nzo);
         g.zb = p.za + (seg_end - g.tile * nzo);
         g.rl0 = max(g.za - D, zmin);
@@ -468,7 +469,7 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                         if (rowmask & (1u << j)) st_row(pout + j * p.nx, out.r[j]);
                 }
             };
-            if (ST7_SPLIT) {   // all in-plane parts first, then the z+1 chain
+            if (SPLIT) {   // all in-plane parts first, then the z+1 chain
 #pragma unroll
                 for (int l = 1; l <= D; ++l) level_A(l);
                 load0();

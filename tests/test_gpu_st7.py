@@ -160,7 +160,8 @@ def test_naive_variant_bitexact(oracle_lib, dtype, T):
 
 @pytest.mark.parametrize("dtype", [np.float32, np.float64])
 def test_autotune_picks_a_depth_and_stays_exact(oracle_lib, dtype):
-    # st_plan_autotune times every depth and keeps the fastest; results are depth-independent
+    # st_plan_autotune: the eq. (3) seed from the measured Gamma, its neighbours timed,
+    # the fastest timed depth kept, and it is a local minimum; results are depth-independent
     nx, ny, nz = 96, 72, 40
     dt = torch.float32 if dtype == np.float32 else torch.float64
     a = stgen.grid7(nx, ny, nz, 11, dtype)
@@ -169,10 +170,17 @@ def test_autotune_picks_a_depth_and_stays_exact(oracle_lib, dtype):
         x = torch.empty(nz, ny, nx, dtype=dt, device="cuda")
         y = torch.empty_like(x)
         d, eta, ms = p.autotune(x, y, 6)
-        assert 1 <= d <= 6 and eta >= 1
-        assert sorted(ms) == list(range(1, len(ms) + 1)) and d in ms
+        assert 1 <= d <= 6 and 1 <= eta
+        assert 1 in ms and 6 in ms and d in ms            # the two Gamma probes and the choice
         assert ms[d] == min(ms.values())
+        for nb in (d - 1, d + 1):                         # a local minimum of the timed depths
+            assert not (1 <= nb <= 6) or nb in ms
         assert p.info()["dim_t_sweep"] == d
+        rep = p.autotune_report(x, y, 6)
+        assert rep["dim_T"] >= 1 and rep["Gamma_eff"] > 0 and rep["eta"] >= 1
+        assert rep["gamma"] == pytest.approx(2 * np.dtype(dtype).itemsize / 7)
+        assert all(s > 0 for s in rep["tile_side"])
+        assert rep["tile_side"][0] < rep["tile_side"][1] < rep["tile_side"][2]
         p.set_bitexact(True)
         x.copy_(torch.from_numpy(a))
         p.st7(x, y, 0.4, 0.1, 9)
