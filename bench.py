@@ -292,7 +292,7 @@ def main():
         p = st.Plan(n, n, nzg, tdt, D)
         p.set_stream(stream)
         if world > 1:
-            st.st_plan_set_dist(p.h, uid, rank, world)
+            p.set_dist(uid, rank, world)
             z0, nzl = st.st_plan_local_slab(p.h)
             g = st.st_plan_ghost_planes(p.h)
         else:

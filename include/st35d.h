@@ -237,7 +237,11 @@ int st_plan_sync(st_plan* plan);
 /* Z-slab distribution (§8(e)): rank owns planes [z0, z0+nz_local) of the
  * global grid (remainder planes go one each to the first ranks).  The
  * 128-byte NCCL unique id comes from rank 0 (broadcast by the caller).
- * nranks == 1 switches distribution off. */
+ * nranks == 1 with a NULL id switches distribution off; with an id it builds
+ * a one-rank communicator that runs the distributed schedule (testing).
+ * The communicator is created with ncclCommInitRankConfig, maxCTAs = 4 (the
+ * exchange overlaps the interior sweep); asynchronous NCCL errors are polled
+ * (ncclCommGetAsyncError) after every run and by st_plan_sync -> ST_ENCCL. */
 int st_plan_set_dist(st_plan* plan, const void* nccl_unique_id, int rank, int nranks);
 
 /* 128-byte NCCL unique id for st_plan_set_dist (call on rank 0, broadcast). */
@@ -246,6 +250,28 @@ int st_nccl_unique_id(void* out128);
 /* Z-slab of `rank` among `nranks`: first global plane and plane count
  * (remainder planes one each to the first ranks).  Host-only. */
 int st_slab_range(int nz, int nranks, int rank, int* z0, int* nz_local);
+
+/* The Z-slab sweep schedule a rank of a distributed plan executes (host-only,
+ * no device needed; st7_run / lbm_d3q19_run run exactly this list, SURVEY
+ * §8(e)).  Buffer coordinates: plane L of a slab buffer is global plane
+ * z0 - g + L, g = dim_T ghost planes per side, owned planes [g, g + nz_local).
+ *   ST_STEP_EXCHANGE: send planes [g, g+depth) of buffer `src` to rank-1 and
+ *     [g+nz_local-depth, g+nz_local) to rank+1; receive the neighbours' into
+ *     [g-depth, g) and [g+nz_local, g+nz_local+depth) (a depth-d sweep
+ *     needs d valid ghost planes per face).  async = 1: overlapped with the
+ *     following ST_STEP_SWEEP steps, up to the next ST_STEP_WAIT.
+ *   ST_STEP_SWEEP: `depth` Jacobi steps from buffer src into buffer 1-src for
+ *     the output planes [z_begin, z_end) (grid_cap = 1: SMs left to NCCL).
+ *   ST_STEP_WAIT: the sweep stream waits for the async exchange.
+ *   ST_STEP_COPY: an even number of sweeps left the result in buffer 0 (`in`).
+ * Buffer 0 is the caller's `in`, 1 its `out`.  overlap = 0 gives the
+ * serialised schedule (ST_OPT_OVERLAP).  Returns the step count (steps may be
+ * NULL to query it) or < 0. */
+enum { ST_STEP_EXCHANGE = 0, ST_STEP_SWEEP = 1, ST_STEP_WAIT = 2, ST_STEP_COPY = 3 };
+typedef struct {
+    int kind, sweep, depth, src, z_begin, z_end, async, grid_cap;
+} st_slab_step;
+int st_slab_schedule(int nz, int nranks, int rank, int dim_T, int T, int overlap, st_slab_step* steps, int max_steps);
 
 /* Loopback distribution on one device (testing): P virtual slabs, ghosts
  * copied with cudaMemcpyAsync instead of NCCL; result identical to P = 1. */

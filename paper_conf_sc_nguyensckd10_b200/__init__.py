@@ -47,6 +47,13 @@ class st_autotune_report(ctypes.Structure):
                 ("capacity", ctypes.c_double * 3), ("tile_side", ctypes.c_int * 3), ("kappa", ctypes.c_double * 3)]
 
 
+class st_slab_step(ctypes.Structure):
+    _fields_ = [(k, ctypes.c_int) for k in ("kind", "sweep", "depth", "src", "z_begin", "z_end", "async_", "grid_cap")]
+
+
+ST_STEP_EXCHANGE, ST_STEP_SWEEP, ST_STEP_WAIT, ST_STEP_COPY = 0, 1, 2, 3
+
+
 class st_blocking(ctypes.Structure):
     _fields_ = [("eta", ctypes.c_int), ("dim_bound", ctypes.c_double), ("dim", ctypes.c_int),
                 ("kappa", ctypes.c_double)]
@@ -58,7 +65,7 @@ EXPORTS = ["st_plan_create", "st7_run", "st13_run", "st27_run", "lbm_d3q19_run",
            "st_plan_set_stream", "st_plan_set_option", "st_plan_set_lbm_lid", "st_plan_set_bitexact", "st_plan_set_variant", "st_plan_autotune", "st_plan_autotune_report", "st_plan_sync",
            "st_plan_set_dist", "st_plan_set_loopback_slabs", "st_plan_ghost_planes", "st_plan_local_slab",
            "st_plan_get_info", "st_plan_last_launches", "st_blocking_model", "st_fig3_step",
-           "st_nccl_unique_id", "st_slab_range"]
+           "st_nccl_unique_id", "st_slab_range", "st_slab_schedule"]
 
 
 def lib() -> ctypes.CDLL:
@@ -97,6 +104,7 @@ def lib() -> ctypes.CDLL:
         "st_fig3_step": ([I, I, I, I, ctypes.POINTER(I), ctypes.POINTER(I)], I),
         "st_nccl_unique_id": ([P], I),
         "st_slab_range": ([I, I, I, ctypes.POINTER(I), ctypes.POINTER(I)], I),
+        "st_slab_schedule": ([I, I, I, I, I, I, ctypes.POINTER(st_slab_step), I], I),
     }
     for name, (args, res) in sig.items():
         if os.environ.get("ST35D_LIB") and not hasattr(L, name):   # A/B build of an older ABI
@@ -266,6 +274,15 @@ def st_slab_range(nz: int, nranks: int, rank: int):
     return z0.value, n.value
 
 
+def st_slab_schedule(nz: int, nranks: int, rank: int, dim_T: int, T: int, overlap: bool = True) -> list:
+    """the Z-slab step list a rank executes (include/st35d.h), as dicts."""
+    n = _check(lib().st_slab_schedule(nz, nranks, rank, dim_T, T, 1 if overlap else 0, None, 0))
+    buf = (st_slab_step * max(n, 1))()
+    _check(lib().st_slab_schedule(nz, nranks, rank, dim_T, T, 1 if overlap else 0, buf, n))
+    return [{"kind": s.kind, "sweep": s.sweep, "depth": s.depth, "src": s.src, "z_begin": s.z_begin,
+             "z_end": s.z_end, "async": s.async_, "grid_cap": s.grid_cap} for s in buf[:n]]
+
+
 def dtype_code(dtype) -> int:
     name = str(dtype)
     if "float32" in name:
@@ -356,7 +373,7 @@ class Plan:
 
     def set_dist(self, unique_id: bytes, rank: int, nranks: int) -> None:
         st_plan_set_dist(self.h, unique_id, rank, nranks)
-        self._nzb = self.shape[0] if nranks == 1 else st_plan_local_slab(self.h)[1] + 2 * st_plan_ghost_planes(self.h)
+        self._nzb = st_plan_local_slab(self.h)[1] + 2 * st_plan_ghost_planes(self.h)   # slab + ghosts
 
     def set_stream(self, stream) -> None:
         st_plan_set_stream(self.h, stream)

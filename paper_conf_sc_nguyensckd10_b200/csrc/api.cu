@@ -17,6 +17,10 @@
 
 using namespace st35d;
 
+// NCCL CTAs per communicator (ncclConfig_t.maxCTAs): the ghost exchange is a few
+// MB per sweep, a handful of CTAs saturate NVLink for it, the rest stay with the sweep
+constexpr int ST_NCCL_MAX_CTAS = 4;
+
 // ----------------------------------------------------------------------------
 // errors
 // ----------------------------------------------------------------------------
@@ -405,11 +409,13 @@ extern "C" int st_plan_set_bitexact(st_plan* p, int on) {
     return ST_OK;
 }
 
+static int poll_nccl(st_plan* p);
+
 extern "C" int st_plan_sync(st_plan* p) {
     if (!p) return fail(ST_EINVAL, "NULL plan");
     CUDA_TRY(cudaStreamSynchronize(p->stream));
     CUDA_TRY(cudaGetLastError());
-    return ST_OK;
+    return poll_nccl(p);
 }
 
 extern "C" int st_plan_ghost_planes(const st_plan* p) { return p ? p->dimT : ST_EINVAL; }
@@ -563,6 +569,21 @@ static int launch7(st_plan* p, const void* src, void* dst, int d, double alpha, 
 // ----------------------------------------------------------------------------
 // ncomp: SoA components of a cell (1 for the 7-point grid, 19 for D3Q19); each
 // component of a slab buffer is nzb consecutive planes.
+// asynchronous NCCL errors (a peer died, a network error) surface as ST_ENCCL
+// at the end of every distributed run and at st_plan_sync
+static int poll_nccl(st_plan* p) {
+#if ST_HAVE_NCCL
+    if (p->dist.mode != Dist::NCCL || !p->dist.nccl_comm || !nccl().commGetAsyncError) return ST_OK;
+    ncclResult_t ae = ncclSuccess;
+    ncclResult_t r = nccl().commGetAsyncError(p->dist.nccl_comm, &ae);
+    if (r != ncclSuccess) return fail(ST_ENCCL, "ncclCommGetAsyncError: %s", nccl().errorString(r));
+    if (ae != ncclSuccess && ae != ncclInProgress) return fail(ST_ENCCL, "NCCL async error: %s", nccl().errorString(ae));
+#else
+    (void)p;
+#endif
+    return ST_OK;
+}
+
 static int exchange_nccl(st_plan* p, void* buf, int d, int ncomp, cudaStream_t st) {
 #if ST_HAVE_NCCL
     Dist& D = p->dist;
@@ -728,48 +749,54 @@ static int run_sweeps(st_plan* p, const std::vector<int>& ds, const void* in, vo
         sv.flags = s.flags; sv.fl2 = s.fl2; sv.single = false; sv.stream = p->stream; sv.grid_cap = cap;
         return sv;
     };
-    int cur = 0;
-    rc = exchange(cur, ds[0], p->stream);   // ghosts of the input
-    if (rc) return rc;
+    // the schedule (dist.h slab_schedule, also exported as st_slab_schedule) is
+    // identical for every slab up to its plane count; run step by step over all slabs
+    int nzl_min = sl[0].nzl;
+    for (auto& s : sl) nzl_min = std::min(nzl_min, s.nzl);
+    std::vector<std::vector<SlabStep>> sched;
+    for (auto& s : sl) sched.push_back(slab_schedule(ds, D.g, s.nzl, nzl_min, overlap_ok));
     const int cap = loop ? 0 : std::max(1, p->sms - 8);   // leave SMs to the NCCL kernels
-    for (size_t k = 0; k < ds.size(); ++k) {
-        const int d = ds[k], dn = k + 1 < ds.size() ? ds[k + 1] : 0;
-        bool split = overlap_ok && dn > 0;
-        for (auto& s : sl) split = split && s.nzl > 2 * dn;
-        if (split) {
-            for (auto& s : sl) {   // boundary planes first
-                rc = launch(s.buf[cur], s.buf[1 - cur], d, view(s, D.g, D.g + dn, 0));
-                if (!rc) rc = launch(s.buf[cur], s.buf[1 - cur], d, view(s, D.g + s.nzl - dn, D.g + s.nzl, 0));
-                if (rc) return rc;
-            }
-            CUDA_TRY(cudaEventRecord(D.ev_b, p->stream));
-            CUDA_TRY(cudaStreamWaitEvent(D.comm, D.ev_b, 0));
-            rc = exchange(1 - cur, dn, D.comm);
-            if (rc) return rc;
-            CUDA_TRY(cudaEventRecord(D.ev_x, D.comm));
-            for (auto& s : sl) {   // interior overlaps the exchange
-                rc = launch(s.buf[cur], s.buf[1 - cur], d, view(s, D.g + dn, D.g + s.nzl - dn, cap));
-                if (rc) return rc;
-            }
-            CUDA_TRY(cudaStreamWaitEvent(p->stream, D.ev_x, 0));
-        } else {
-            for (auto& s : sl) {
-                rc = launch(s.buf[cur], s.buf[1 - cur], d, view(s, D.g, D.g + s.nzl, 0));
-                if (rc) return rc;
-            }
-            if (dn > 0) {
-                rc = exchange(1 - cur, dn, p->stream);
-                if (rc) return rc;
-            }
+    int cur = 0;
+    for (size_t i = 0; i < sched[0].size(); ++i) {
+        const SlabStep& st0 = sched[0][i];
+        switch (st0.kind) {
+            case SlabStep::EXCHANGE:
+                if (st0.async) {
+                    CUDA_TRY(cudaEventRecord(D.ev_b, p->stream));
+                    CUDA_TRY(cudaStreamWaitEvent(D.comm, D.ev_b, 0));
+                    rc = exchange(st0.src, st0.depth, D.comm);
+                    if (rc) return rc;
+                    CUDA_TRY(cudaEventRecord(D.ev_x, D.comm));
+                } else {
+                    rc = exchange(st0.src, st0.depth, p->stream);
+                    if (rc) return rc;
+                }
+                break;
+            case SlabStep::SWEEP:
+                for (size_t k = 0; k < sl.size(); ++k) {
+                    const SlabStep& stp = sched[k][i];
+                    rc = launch(sl[k].buf[stp.src], sl[k].buf[1 - stp.src], stp.depth,
+                                view(sl[k], stp.z_begin, stp.z_end, stp.grid_cap ? cap : 0));
+                    if (rc) return rc;
+                }
+                cur = 1 - st0.src;
+                break;
+            case SlabStep::WAIT:
+                CUDA_TRY(cudaStreamWaitEvent(p->stream, D.ev_x, 0));
+                break;
+            case SlabStep::COPY:
+                cur = 0;
+                break;
         }
-        cur ^= 1;
     }
+    rc = poll_nccl(p);
+    if (rc) return rc;
     if (loop) {
         for (auto& s : D.slabs) {   // gather owned planes
             rc = slab_copy(p, out, cur == 0 ? s.buf[0] : s.buf[1], s.z0 - D.g, s.nzb, s.z0, s.nzl, ncomp, false);
             if (rc) return rc;
         }
-    } else if (cur == 0) {   // even number of sweeps: the result is in `in`
+    } else if (cur == 0) {   // even number of sweeps (the schedule's COPY): the result is in `in`
         CUDA_TRY(cudaMemcpyAsync(out, in, (size_t)ncomp * D.nzb * pb, cudaMemcpyDeviceToDevice, p->stream));
     }
     return ST_OK;
@@ -1286,6 +1313,8 @@ bool st35d::NcclApi::load() {
     if (!h) return false;
     getUniqueId = reinterpret_cast<decltype(getUniqueId)>(dlsym(h, "ncclGetUniqueId"));
     commInitRank = reinterpret_cast<decltype(commInitRank)>(dlsym(h, "ncclCommInitRank"));
+    commInitRankConfig = reinterpret_cast<decltype(commInitRankConfig)>(dlsym(h, "ncclCommInitRankConfig"));
+    commGetAsyncError = reinterpret_cast<decltype(commGetAsyncError)>(dlsym(h, "ncclCommGetAsyncError"));
     commDestroy = reinterpret_cast<decltype(commDestroy)>(dlsym(h, "ncclCommDestroy"));
     send = reinterpret_cast<decltype(send)>(dlsym(h, "ncclSend"));
     recv = reinterpret_cast<decltype(recv)>(dlsym(h, "ncclRecv"));
@@ -1340,11 +1369,30 @@ extern "C" int st_slab_range(int nz, int nranks, int rank, int* z0, int* nz_loca
     return ST_OK;
 }
 
+extern "C" int st_slab_schedule(int nz, int nranks, int rank, int dim_T, int T, int overlap, st_slab_step* steps,
+                                int max_steps) {
+    if (nz < 1 || nranks < 1 || rank < 0 || rank >= nranks || nz < nranks || dim_T < 1 || T < 0)
+        return fail(ST_EINVAL, "slab schedule arguments");
+    if (nranks > 1 && nz / nranks < dim_T) return fail(ST_EINVAL, "slabs thinner than dim_T");
+    int z0 = 0, nzl = 0;
+    slab_range(nz, nranks, rank, z0, nzl);
+    const std::vector<SlabStep> v = slab_schedule(sweep_depths(T, dim_T), dim_T, nzl, nz / nranks, overlap != 0);
+    if (steps) {
+        if (max_steps < (int)v.size()) return fail(ST_EINVAL, "schedule has %zu steps, room for %d", v.size(), max_steps);
+        for (size_t i = 0; i < v.size(); ++i)
+            steps[i] = st_slab_step{v[i].kind, v[i].sweep, v[i].depth, v[i].src, v[i].z_begin, v[i].z_end, v[i].async,
+                                    v[i].grid_cap};
+    }
+    return (int)v.size();
+}
+
 extern "C" int st_plan_set_dist(st_plan* p, const void* uid, int rank, int nranks) {
     if (!p) return fail(ST_EINVAL, "NULL plan");
     if (nranks < 1 || rank < 0 || rank >= nranks) return fail(ST_EINVAL, "rank %d of %d", rank, nranks);
     CUDA_TRY(cudaStreamSynchronize(p->stream));
-    if (nranks == 1) { p->dist.init_single(p->nz); return ST_OK; }
+    if (nranks == 1 && !uid) { p->dist.init_single(p->nz); return ST_OK; }   // distribution off
+    // (nranks == 1 with an id: a one-rank NCCL communicator running the full
+    // distributed schedule -- the single-GPU test of the NCCL path)
     const int g = p->dimT;
     int z0 = 0, nzl = 0;
     slab_range(p->nz, nranks, rank, z0, nzl);
@@ -1356,8 +1404,20 @@ extern "C" int st_plan_set_dist(st_plan* p, const void* uid, int rank, int nrank
     ncclUniqueId id;
     memcpy(&id, uid, sizeof id);
     ncclComm_t comm = nullptr;
-    ncclResult_t r = nccl().commInitRank(&comm, nranks, id, rank);
-    if (r != ncclSuccess) return fail(ST_ENCCL, "ncclCommInitRank: %s", nccl().errorString(r));
+    ncclResult_t r;
+    if (nccl().commInitRankConfig) {
+        // cap NCCL's CTAs so the exchange overlaps the interior sweep, which
+        // leaves the same SMs free (run_sweeps grid cap)
+        ncclConfig_t cfg = NCCL_CONFIG_INITIALIZER;
+        cfg.blocking = 1;
+        cfg.minCTAs = 1;
+        cfg.maxCTAs = ST_NCCL_MAX_CTAS;
+        r = nccl().commInitRankConfig(&comm, nranks, id, rank, &cfg);
+        if (r != ncclSuccess) return fail(ST_ENCCL, "ncclCommInitRankConfig: %s", nccl().errorString(r));
+    } else {
+        r = nccl().commInitRank(&comm, nranks, id, rank);
+        if (r != ncclSuccess) return fail(ST_ENCCL, "ncclCommInitRank: %s", nccl().errorString(r));
+    }
     Dist& D = p->dist;
     D.mode = Dist::NCCL; D.nccl_comm = comm;
     D.nz = p->nz; D.P = nranks; D.rank = rank; D.g = g; D.z0 = z0; D.nzl = nzl; D.nzb = nzl + 2 * g;

@@ -1,11 +1,14 @@
-"""Multi-process (world_size 2, gloo, CPU) check of the Z-slab decomposition
-host logic of §8(e): slab ranges from the library (st_slab_range, host-only),
-dim_T-deep ghost planes exchanged with the neighbour rank before every
-sweep, each rank advancing only its slab.  The compute here is the CPU oracle
-on the slab buffer (its fixed buffer edges are exactly the ghost-zone
-argument of P:216: after d steps only planes >= d away from the buffer edge
-are valid), so the test checks the decomposition and exchange schedule the
-NCCL transport uses, independently of the GPU."""
+"""Multi-process (world_size 2 and 3, gloo, CPU) check of the Z-slab
+decomposition of §8(e) as the library runs it: every rank executes the step
+list the library itself builds for st7_run / lbm_d3q19_run
+(st_slab_schedule, host-only: ghosts of the input, boundary planes first,
+the exchange of the next sweep's ghosts overlapped with the interior sweep,
+waits, the final copy), with gloo send/recv as the transport and the CPU
+oracle as the per-step compute on the slab buffer (its fixed buffer edges are
+the ghost-zone argument of P:216: after d steps only planes >= d away from an
+artificial buffer edge are valid).  The gathered result must equal the
+single-domain oracle bit for bit, so a wrong plane range, ghost depth,
+buffer parity or wait in the library's schedule fails it."""
 import os
 import socket
 
@@ -26,12 +29,6 @@ def _free_port():
     return p
 
 
-def _sweep_depths(T, D):
-    S = -(-T // D)
-    q, rem = divmod(T, S)
-    return [q + (1 if s < rem else 0) for s in range(S)]
-
-
 def _worker(rank, world, port, kind, q):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
@@ -42,64 +39,89 @@ def _worker(rank, world, port, kind, q):
         nx, ny, nz, D, T = 20, 18, 27, 3, 8
         z0, nzl = st.st_slab_range(nz, world, rank)
         g = D
-        lo, hi = max(0, z0 - g), min(nz, z0 + nzl + g)     # buffer planes (clipped at the lattice)
-        own = slice(z0 - lo, z0 - lo + nzl)
+        nzb = nzl + 2 * g
+        steps = st.st_slab_schedule(nz, world, rank, D, T, overlap=True)
+        # buffer plane L <-> global z0 - g + L; planes outside the grid stay zero (never valid)
+        lo, hi = max(0, z0 - g), min(nz, z0 + nzl + g)
+        Lmin, Lmax = lo - (z0 - g), hi - (z0 - g)
         if kind == "st7":
             full = stgen.grid7(nx, ny, nz, 41, np.float64)
-            buf = full[lo:hi].copy()
-            comp = lambda b: b[None]                           # noqa: E731
+            bufs = [np.zeros((1, nzb, ny, nx)), np.zeros((1, nzb, ny, nx))]
+            bufs[0][0, Lmin:Lmax] = full[lo:hi]
         else:
             flags_full = stgen.cavity_flags(nx, ny, nz)
             full = stgen.lbm_random(nx, ny, nz, 42, np.float64)
-            buf = full[:, lo:hi].copy()
+            bufs = [np.zeros((19, nzb, ny, nx)), np.zeros((19, nzb, ny, nx))]
+            bufs[0][:, Lmin:Lmax] = full[:, lo:hi]
             fl = flags_full[lo:hi].copy()
-            comp = lambda b: b                                 # noqa: E731
-        for d in _sweep_depths(T, D):
-            # ghost exchange: my d planes next to each face <-> neighbour's
-            c = comp(buf)
-            reqs = []
-            if rank > 0:
-                send_lo = torch.from_numpy(np.ascontiguousarray(c[:, z0 - lo:z0 - lo + d]))
-                recv_lo = torch.empty_like(send_lo)
-                reqs += [dist.isend(send_lo, rank - 1), dist.irecv(recv_lo, rank - 1)]
-            if rank < world - 1:
-                e = z0 - lo + nzl
-                send_hi = torch.from_numpy(np.ascontiguousarray(c[:, e - d:e]))
-                recv_hi = torch.empty_like(send_hi)
-                reqs += [dist.isend(send_hi, rank + 1), dist.irecv(recv_hi, rank + 1)]
-            for r in reqs:
-                r.wait()
-            if rank > 0:
-                c[:, z0 - lo - d:z0 - lo] = recv_lo.numpy()
-            if rank < world - 1:
-                e = z0 - lo + nzl
-                c[:, e:e + d] = recv_hi.numpy()
-            # d steps on the slab buffer; only owned planes are kept valid
+
+        def compute(src, depth):   # the oracle on the part of the buffer inside the grid
             if kind == "st7":
-                buf = oracle.st7(buf, 0.4, 0.1, d)
-            else:
-                buf = oracle.lbm(buf, fl, 1.6, d)
-        owned = buf[own] if kind == "st7" else buf[:, own]
+                return oracle.st7(np.ascontiguousarray(src[0, Lmin:Lmax]), 0.4, 0.1, depth)[None]
+            return oracle.lbm(np.ascontiguousarray(src[:, Lmin:Lmax]), fl, 1.6, depth)
+
+        pending = []
+
+        def start_exchange(b, d):
+            c = bufs[b]
+            ops = []
+            if rank > 0:
+                send = torch.from_numpy(np.ascontiguousarray(c[:, g:g + d]))
+                recv = torch.empty_like(send)
+                ops.append((dist.isend(send, rank - 1), dist.irecv(recv, rank - 1), b, g - d, g, recv))
+            if rank < world - 1:
+                e = g + nzl
+                send = torch.from_numpy(np.ascontiguousarray(c[:, e - d:e]))
+                recv = torch.empty_like(send)
+                ops.append((dist.isend(send, rank + 1), dist.irecv(recv, rank + 1), b, e, e + d, recv))
+            return ops
+
+        def finish(ops):
+            for s_, r_, b, z_a, z_b, recv in ops:
+                s_.wait()
+                r_.wait()
+                bufs[b][:, z_a:z_b] = recv.numpy()
+
+        result = None
+        for stp in steps:
+            if stp["kind"] == st.ST_STEP_EXCHANGE:
+                ops = start_exchange(stp["src"], stp["depth"])
+                if stp["async"]:
+                    pending = ops       # completes at the next WAIT
+                else:
+                    finish(ops)
+            elif stp["kind"] == st.ST_STEP_SWEEP:
+                out = compute(bufs[stp["src"]], stp["depth"])
+                za, zb = stp["z_begin"], stp["z_end"]
+                assert g <= za <= zb <= g + nzl
+                bufs[1 - stp["src"]][:, za:zb] = out[:, za - Lmin:zb - Lmin]
+                result = 1 - stp["src"]
+            elif stp["kind"] == st.ST_STEP_WAIT:
+                finish(pending)
+                pending = []
+            elif stp["kind"] == st.ST_STEP_COPY:
+                result = 0
+        assert not pending
+        owned = bufs[result][:, g:g + nzl]
         parts = [None] * world
         dist.all_gather_object(parts, (z0, owned))
         if rank == 0:
+            got = np.concatenate([p[1] for p in sorted(parts, key=lambda t: t[0])], axis=1)
             if kind == "st7":
-                ref = oracle.st7(full, 0.4, 0.1, T)
-                got = np.concatenate([p[1] for p in sorted(parts, key=lambda t: t[0])], axis=0)
+                ok = np.array_equal(got[0], oracle.st7(full, 0.4, 0.1, T))
             else:
-                ref = oracle.lbm(full, flags_full, 1.6, T)
-                got = np.concatenate([p[1] for p in sorted(parts, key=lambda t: t[0])], axis=1)
-            q.put(bool(np.array_equal(got, ref)))
+                ok = np.array_equal(got, oracle.lbm(full, flags_full, 1.6, T))
+            q.put(bool(ok))
     finally:
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("kind", ["st7", "lbm"])
-def test_zslab_world2_gloo(kind):
+@pytest.mark.parametrize("kind,world", [("st7", 2), ("lbm", 2), ("st7", 3)])
+def test_zslab_schedule_gloo(kind, world):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, kind, q)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, kind, q)) for r in range(world)]
     for p in procs:
         p.start()
     for p in procs:
@@ -117,3 +139,32 @@ def test_slab_ranges():
         assert all(ranges[i][0] + ranges[i][1] == ranges[i + 1][0] for i in range(P - 1))
         assert max(n for _, n in ranges) - min(n for _, n in ranges) <= 1
         assert [n for _, n in ranges] == sorted([n for _, n in ranges], reverse=True)
+
+
+def test_schedule_structure():
+    # host-only properties of the library's schedule: every owned plane is written by
+    # exactly one SWEEP step per sweep, the ghost depth of an exchange equals the depth
+    # of the sweep that reads it, async exchanges are closed by a WAIT before the next sweep
+    import paper_conf_sc_nguyensckd10_b200 as st
+    for nz, P, D, T, ov in ((512, 8, 4, 100, True), (27, 2, 3, 8, False), (100, 7, 2, 9, True), (64, 4, 1, 6, True)):
+        for r in range(P):
+            z0, nzl = st.st_slab_range(nz, P, r)
+            steps = st.st_slab_schedule(nz, P, r, D, T, ov)
+            cover, open_async, ghost = {}, False, {}
+            for s in steps:
+                if s["kind"] == st.ST_STEP_EXCHANGE:
+                    ghost[s["src"]] = s["depth"]
+                    open_async = bool(s["async"])
+                elif s["kind"] == st.ST_STEP_SWEEP:
+                    assert 1 <= s["depth"] <= D
+                    if s["sweep"] not in cover:    # the ghosts this sweep reads are as deep as the sweep
+                        assert ghost.get(s["src"]) == s["depth"] or P == 1
+                    cover.setdefault(s["sweep"], []).extend(range(s["z_begin"], s["z_end"]))
+                elif s["kind"] == st.ST_STEP_WAIT:
+                    assert open_async
+                    open_async = False
+            assert not open_async
+            for k, planes in cover.items():
+                assert sorted(planes) == list(range(D, D + nzl)), (nz, P, r, k)
+            depths = [s["depth"] for s in steps if s["kind"] == st.ST_STEP_SWEEP and s["z_begin"] == D]
+            assert sum(depths) == T

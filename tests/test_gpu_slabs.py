@@ -72,3 +72,51 @@ def test_slab_too_thin():
     with st.Plan(64, 64, 16, torch.float32, 4) as p:
         with pytest.raises(st.StError):
             st.st_plan_set_loopback_slabs(p.h, 8)   # 2-plane slabs < dim_T
+
+
+@pytest.mark.parametrize("kind", ["st7", "lbm"])
+@pytest.mark.parametrize("overlap", [1, 0])
+def test_nccl_one_rank_communicator(oracle_lib, kind, overlap):
+    # the NCCL transport path on one GPU: st_plan_set_dist with an id and one rank builds a
+    # communicator (ncclCommInitRankConfig, maxCTAs) and runs the distributed schedule --
+    # slab buffers with dim_T ghost planes per side, boundary sweeps, the grouped
+    # send/recv (no peers) on the side stream, the interior sweep, the wait, the async
+    # error poll -- and must still equal the oracle bit for bit
+    dim_T, T = 3, 8
+    uid = st.st_nccl_unique_id()
+    if kind == "st7":
+        nx, ny, nz = 64, 40, 30
+        a = stgen.grid7(nx, ny, nz, 33, np.float32)
+        with st.Plan(nx, ny, nz, torch.float32, dim_T) as p:
+            p.set_bitexact(True)
+            p.set_option(st.ST_OPT_OVERLAP, overlap)
+            p.set_dist(uid, 0, 1)
+            g = st.st_plan_ghost_planes(p.h)
+            assert st.st_plan_local_slab(p.h) == (0, nz)
+            buf = np.zeros((nz + 2 * g, ny, nx), np.float32)
+            buf[g:g + nz] = a
+            x = torch.from_numpy(buf).cuda()
+            y = torch.zeros_like(x)
+            p.st7(x, y, 0.4, 0.1, T)
+            p.sync()
+            got = y.cpu().numpy()[g:g + nz]
+        assert np.array_equal(got, oracle_lib.st7(a, 0.4, 0.1, T))
+    else:
+        nx, ny, nz = 32, 24, 20
+        flags = stgen.cavity_flags(nx, ny, nz)
+        f0 = stgen.lbm_random(nx, ny, nz, 34, np.float32)
+        with st.Plan(nx, ny, nz, torch.float32, 1) as p:
+            p.set_bitexact(True)
+            p.set_option(st.ST_OPT_OVERLAP, overlap)
+            p.set_dist(uid, 0, 1)
+            g = st.st_plan_ghost_planes(p.h)
+            buf = np.zeros((19, nz + 2 * g, ny, nx), np.float32)
+            buf[:, g:g + nz] = f0
+            fl = np.full((nz + 2 * g, ny, nx), stgen.WALL, np.uint8)
+            fl[g:g + nz] = flags
+            x = torch.from_numpy(buf).cuda()
+            y = torch.zeros_like(x)
+            p.lbm(x, y, 1.6, T, torch.from_numpy(fl).cuda())
+            p.sync()
+            got = y.cpu().numpy()[:, g:g + nz]
+        assert np.array_equal(got, oracle_lib.lbm(f0, flags, 1.6, T))
