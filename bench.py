@@ -131,9 +131,11 @@ def n_sweeps(T, D):
 
 
 def load_traffic(key):
+    """dram__bytes_read.sum + dram__bytes_write.sum per launch of that kernel (ncu, profiles/)"""
     try:
         with open(TRAFFIC_PATH) as fh:
-            return json.load(fh).get(key)
+            v = json.load(fh).get(key)
+        return v.get("per_launch_bytes") if isinstance(v, dict) else v
     except Exception:
         return None
 

@@ -5,6 +5,6 @@ mkdir -p gpurun_out/ladder
 M=gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,dram__throughput.avg.pct_of_peak_sustained_elapsed,sm__inst_executed_pipe_fma.sum,sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active,sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active,smsp__issue_active.avg.pct_of_peak_sustained_active,sm__sass_thread_inst_executed_op_ffma_pred_on.sum,sm__sass_thread_inst_executed_op_fadd_pred_on.sum,sm__sass_thread_inst_executed_op_fmul_pred_on.sum,sm__sass_thread_inst_executed_op_ffma2_pred_on.sum,sm__sass_thread_inst_executed_op_fadd2_pred_on.sum,sm__sass_thread_inst_executed_op_fmul2_pred_on.sum,sm__inst_executed_pipe_fmaheavy.sum,sm__inst_executed_pipe_fmalite.sum,sm__pipe_fmaheavy_cycles_active.avg.pct_of_peak_sustained_active,sm__pipe_fmalite_cycles_active.avg.pct_of_peak_sustained_active,sm__sass_thread_inst_executed_op_dfma_pred_on.sum,sm__sass_thread_inst_executed_op_dadd_pred_on.sum,sm__sass_thread_inst_executed_op_dmul_pred_on.sum,l1tex__data_pipe_lsu_wavefronts_mem_shared.sum,sm__cycles_elapsed.avg.per_second,smsp__inst_executed.sum,launch__registers_per_thread,sm__warps_active.avg.pct_of_peak_sustained_active
 for b in naive spatial 4d onerow level twophase; do
   k=regex:st7_35d; [ $b = naive ] && k=regex:st7_naive
-  timeout 600 ncu --metrics $M --clock-control none -k $k -s 3 -c 1 --csv python tools/prof_bar.py $b > gpurun_out/ladder/$b.csv 2>gpurun_out/ladder/$b.err
+  timeout 600 ncu --metrics $M --clock-control none -k $k -s 1 -c 1 --csv python tools/prof_bar.py $b > gpurun_out/ladder/$b.csv 2>gpurun_out/ladder/$b.err
   echo "$b rc=$?"
 done
