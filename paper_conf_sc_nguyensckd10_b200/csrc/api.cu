@@ -88,6 +88,7 @@ struct Geo7 {
     int ey = 0, ly_last = 0, oy0_last = 0;   // y placement (St7Params)
     int maxt = 0;                            // threads of the kernel variant (>= threads launched)
     int minb = 1;                            // CTAs per SM of the variant
+    int vxk = 0;                             // points per thread row (0: the dtype's 16-byte vector)
     size_t smem = 0;
     double kappa = 0;
     St7LaunchFn fn = nullptr;
@@ -142,22 +143,30 @@ static bool lbm_use_push(const st_plan* p);
 // level in registers and fits 256 threads up to dim_T = 4 without spills;
 // deeper sweeps use VY = 2 (half the window per thread, twice the exchange
 // traffic per point).  ST_OPT_ST7_VARIANT overrides (A/B).
-static void variant_for(const st_plan* p, int d, int& vy, int& nt, int& minb) {
+static void variant_for(const st_plan* p, int d, int& vy, int& nt, int& minb, int& vx) {
     minb = 1;
+    vx = 0;
     if (p->opt_st7_variant) {
-        vy = p->opt_st7_variant / 1000 % 10; nt = p->opt_st7_variant % 1000; minb = std::max(1, p->opt_st7_variant / 10000);
+        const int v = p->opt_st7_variant;
+        vy = v / 1000 % 10; nt = v % 1000; minb = std::max(1, v / 10000 % 10); vx = v / 100000;
         return;
     }
     vy = d <= 4 ? 4 : 2;
     nt = 256;
+    // FP32 dim_T <= 4 on grids with long z-runs per CTA (~64x60 tiles x planes over
+    // the SMs): the narrow layout (2 points per thread row, no constructed pairs)
+    // with 16 warps per SM; measured on B200 512^3 dim_T 4: 1600 vs 1385 Gupd/s,
+    // while 256^3 (43 planes per CTA, restart-bound) prefers 8 wide warps (1239 vs 1171)
+    const double run = (double)p->nx * p->ny / (64.0 * 60.0) * p->dist.nzl / std::max(1, p->sms);
+    if (p->dtype == ST_F32 && d <= 4 && run >= 150.0) { vx = 2; nt = 512; return; }
     // FP64 (2 doubles per 16-byte vector, 32 threads per tile row): VY = 2 gives
     // 16-row tiles, too short for dim_T >= 7 (written rows 16 - 2 dim_T)
-    if (p->dtype == ST_F64) vy = (d <= 3 || d >= 7) ? 4 : 2;
+    if (p->dtype == ST_F64) vy = (d <= 4 || d >= 7) ? 4 : 2;   // measured 256^3 dim_T 4: VY 4 699, VY 2 385 Gupd/s
 }
 
-static St7LaunchFn lookup7(st_dtype dt, bool exact, int d, int vy, int nt, int minb) {
-    if (dt == ST_F32) return exact ? st7_lookup_f32_exact(d, vy, nt, minb) : st7_lookup_f32_fast(d, vy, nt, minb);
-    return exact ? st7_lookup_f64_exact(d, vy, nt, minb) : st7_lookup_f64_fast(d, vy, nt, minb);
+static St7LaunchFn lookup7(st_dtype dt, bool exact, int d, int vy, int nt, int minb, int vx = 0) {
+    if (dt == ST_F32) return exact ? st7_lookup_f32_exact(d, vy, nt, minb, vx) : st7_lookup_f32_fast(d, vy, nt, minb, vx);
+    return exact ? st7_lookup_f64_exact(d, vy, nt, minb, vx) : st7_lookup_f64_fast(d, vy, nt, minb, vx);
 }
 
 // CTAs per SM of a variant (minb 9 = the ladder's level-by-level kernel, one per SM)
@@ -193,13 +202,17 @@ static void place_y(Geo7& g, int ny, int d, int R = 1) {
 
 static int plan7(st_plan* p, int d, int nzo, Geo7& g) {
     g.d = d;
-    g.VX = p->dtype == ST_F32 ? 4 : 2;
-    g.NTX = p->dtype == ST_F32 ? 16 : 32;
+    int ntmax = 0, vx = 0;
+    variant_for(p, d, g.VY, ntmax, g.minb, vx);
+    g.vxk = vx;
+    g.VX = vx ? vx : (p->dtype == ST_F32 ? 4 : 2);
+    g.NTX = 64 / g.VX;
     g.TX = g.NTX * g.VX;
-    int ntmax = 0;
-    variant_for(p, d, g.VY, ntmax, g.minb);
-    g.hx = (d + g.VX - 1) / g.VX * g.VX;
-    g.wx = (g.TX - g.hx - d) & ~(g.VX - 1);
+    // TMA boxes must start on a 16-byte boundary: halo and written width in
+    // 16-byte units (4 FP32 / 2 FP64 points) whatever the points per thread
+    const int al16 = (int)(16 / esize(p->dtype));
+    g.hx = (d + al16 - 1) / al16 * al16;
+    g.wx = (g.TX - g.hx - d) & ~(al16 - 1);
     if (g.wx < g.VX) return fail(ST_EUNSUPPORTED, "dim_T %d too deep for the %d-wide tile of this build", d, g.TX);
     g.tiles_x = (p->nx + g.wx - 1) / g.wx;
     // tile height: the thread-row count (<= the variant's threads) that loads
@@ -229,7 +242,7 @@ static int plan7(st_plan* p, int d, int nzo, Geo7& g) {
     const long long work = (long long)g.tiles_x * g.tiles_y * nzo;
     g.grid = (int)std::min<long long>((long long)p->sms * ctas_per_sm(g), std::max<long long>(work, 1));
     g.kappa = (double)g.tiles_x * g.TX * g.tiles_y * g.TY / ((double)p->nx * p->ny);
-    g.fn = lookup7(p->dtype, p->exact, d, g.VY, ntmax, g.minb);
+    g.fn = lookup7(p->dtype, p->exact, d, g.VY, ntmax, g.minb, g.vxk);
     if (!g.fn) return fail(ST_EUNSUPPORTED, "no kernel for dim_T %d (VY %d, %d threads)", d, g.VY, ntmax);
     g.maxt = ntmax;
     return ST_OK;
@@ -238,7 +251,7 @@ static int plan7(st_plan* p, int d, int nzo, Geo7& g) {
 static int get_geo7(st_plan* p, int d, int nzo, Geo7*& out) {
     auto it = p->geo7.find(d);
     if (it == p->geo7.end() ||
-        it->second.fn != lookup7(p->dtype, p->exact, d, it->second.VY, it->second.maxt, it->second.minb)) {
+        it->second.fn != lookup7(p->dtype, p->exact, d, it->second.VY, it->second.maxt, it->second.minb, it->second.vxk)) {
         Geo7 g;
         int rc = plan7(p, d, nzo, g);
         if (rc) return rc;
@@ -394,7 +407,8 @@ extern "C" int st_plan_set_option(st_plan* p, int option, int value) {
             p->opt_zchunk = value;
             return ST_OK;
         case ST_OPT_ST7_VARIANT:
-            if (value != 0 && !lookup7(p->dtype, p->exact, 1, value / 1000 % 10, value % 1000, std::max(1, value / 10000)))
+            if (value != 0 && !lookup7(p->dtype, p->exact, 1, value / 1000 % 10, value % 1000,
+                                       std::max(1, value / 10000 % 10), value / 100000))
                 return fail(ST_EINVAL, "ST_OPT_ST7_VARIANT %d is not compiled", value);
             p->opt_st7_variant = value;
             p->geo7.clear();
@@ -450,7 +464,8 @@ extern "C" int st_plan_get_info(const st_plan* p, int lbm, st_plan_info* info) {
     const Geo7& g = *gp;
     info->tile_x = g.TX; info->tile_y = g.TY; info->out_x = g.wx; info->out_y = g.wy;
     info->tiles_x = g.tiles_x; info->tiles_y = g.tiles_y; info->ctas = g.grid; info->threads = g.threads;
-    info->smem_bytes = (int)g.smem; info->kappa = g.kappa; info->kernel = g.minb * 10000 + g.VY * 1000 + g.maxt;
+    info->smem_bytes = (int)g.smem; info->kappa = g.kappa;
+    info->kernel = g.vxk * 100000 + g.minb * 10000 + g.VY * 1000 + g.maxt;
     info->dim_t_sweep = p->dimK;
     info->ring = g.ring;
     return ST_OK;
@@ -1419,6 +1434,7 @@ extern "C" int st_plan_set_dist(st_plan* p, const void* uid, int rank, int nrank
         if (r != ncclSuccess) return fail(ST_ENCCL, "ncclCommInitRank: %s", nccl().errorString(r));
     }
     Dist& D = p->dist;
+    p->geo7.clear();   // the kernel variant depends on the local slab
     D.mode = Dist::NCCL; D.nccl_comm = comm;
     D.nz = p->nz; D.P = nranks; D.rank = rank; D.g = g; D.z0 = z0; D.nzl = nzl; D.nzb = nzl + 2 * g;
     D.nranks = nranks;

@@ -31,11 +31,11 @@ inline cudaError_t launch_pdl(bool pdl, K kernel, int grid, int threads, size_t 
 using St7LaunchFn = cudaError_t (*)(const CUtensorMap* map, const St7Params& p, int grid, int threads,
                                     size_t smem, cudaStream_t s);
 
-// returns nullptr if (D, VY, NT, MINB) is not compiled
-St7LaunchFn st7_lookup_f32_fast(int D, int VY, int NT, int MINB);
-St7LaunchFn st7_lookup_f32_exact(int D, int VY, int NT, int MINB);
-St7LaunchFn st7_lookup_f64_fast(int D, int VY, int NT, int MINB);
-St7LaunchFn st7_lookup_f64_exact(int D, int VY, int NT, int MINB);
+// returns nullptr if (D, VY, NT, MINB, VX) is not compiled (VX 0: the dtype's 16-byte vector)
+St7LaunchFn st7_lookup_f32_fast(int D, int VY, int NT, int MINB, int VX);
+St7LaunchFn st7_lookup_f32_exact(int D, int VY, int NT, int MINB, int VX);
+St7LaunchFn st7_lookup_f64_fast(int D, int VY, int NT, int MINB, int VX);
+St7LaunchFn st7_lookup_f64_exact(int D, int VY, int NT, int MINB, int VX);
 
 // radius-2 (13-point star) sweep (st13_kernel.cuh); nullptr if (D, VY) is not compiled
 struct St13Params;

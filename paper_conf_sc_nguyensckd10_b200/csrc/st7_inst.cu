@@ -28,10 +28,11 @@ namespace ST_UNIT_NS {
 using TT = ST_T;
 constexpr int NTX = sizeof(TT) == 4 ? 16 : 32;   // threads across the 64-point tile row
 
-template <int D, int VY, int NT, int MINB, bool SPLIT = true>
+template <int D, int VY, int NT, int MINB, bool SPLIT = true, int VX = 0>
 cudaError_t launch(const CUtensorMap* map, const St7Params& p, int grid, int threads, size_t smem, cudaStream_t s) {
-    auto k = st7_35d_kernel<TT, D, NTX, VY, ST_EXACT != 0, NT, MINB, SPLIT>;
-    if (threads > NT || threads % NTX) return cudaErrorInvalidValue;
+    constexpr int NTXK = VX ? 64 / VX : NTX;
+    auto k = st7_35d_kernel<TT, D, NTXK, VY, ST_EXACT != 0, NT, MINB, SPLIT, VX>;
+    if (threads > NT || threads % NTXK) return cudaErrorInvalidValue;
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     return launch_pdl(p.pdl != 0, k, grid, threads, smem, s, *map, p);
@@ -51,13 +52,13 @@ St7LaunchFn pick(int D) {
         default: return nullptr;
     }
 }
-template <int VY, int NT, int MINB, bool SPLIT = true>
+template <int VY, int NT, int MINB, bool SPLIT = true, int VX = 0>
 St7LaunchFn pick4(int D) {   // shallow sweeps only (register cap 65536 / (NT * MINB))
     switch (D) {
-        case 1: return launch<1, VY, NT, MINB, SPLIT>;
-        case 2: return launch<2, VY, NT, MINB, SPLIT>;
-        case 3: return launch<3, VY, NT, MINB, SPLIT>;
-        case 4: return launch<4, VY, NT, MINB, SPLIT>;
+        case 1: return launch<1, VY, NT, MINB, SPLIT, VX>;
+        case 2: return launch<2, VY, NT, MINB, SPLIT, VX>;
+        case 3: return launch<3, VY, NT, MINB, SPLIT, VX>;
+        case 4: return launch<4, VY, NT, MINB, SPLIT, VX>;
         default: return nullptr;
     }
 }
@@ -70,7 +71,15 @@ using namespace ST_UNIT_NS;
 // compiled variants (rows per thread VY, threads per CTA NT, CTAs per SM MINB;
 // MINB = 9: the level-by-level round order of the ablation ladder): see
 // variant_for in api.cu
-St7LaunchFn ST_FN(int D, int VY, int NT, int MINB) {
+St7LaunchFn ST_FN(int D, int VY, int NT, int MINB, int VX) {
+    if constexpr (sizeof(TT) == 4) {
+        if (VX == 2) {   // narrow FP32 layout: 32 threads x 2 points per tile row
+            if (MINB == 1 && VY == 4 && NT == 512) return pick4<4, 512, 1, true, 2>(D);
+            if (MINB == 1 && VY == 4 && NT == 256) return pick4<4, 256, 1, true, 2>(D);
+            return nullptr;
+        }
+    }
+    if (VX != 0 && VX != (sizeof(TT) == 4 ? 4 : 2)) return nullptr;
 #if !ST_EXACT
     if (sizeof(TT) == 4 && MINB == 9 && VY == 4 && NT == 256) return pick4<4, 256, 1, false>(D);   // ladder: no phase split
     if (sizeof(TT) == 4 && MINB == 1 && VY == 1 && NT == 256) return pick4<1, 256, 1>(D);           // ladder: one row per thread

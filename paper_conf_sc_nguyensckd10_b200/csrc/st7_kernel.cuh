@@ -77,37 +77,62 @@ struct St7Params {
 //    sm_100a instructions (FADD2 x4, FMUL2, FFMA2 x2) for 2 points.
 //  * FP64: two scalars (no packed DP form).
 // ---------------------------------------------------------------------------
-template <typename T> struct Rw;
-template <> struct Rw<float> { float2 a, b; };
-template <> struct Rw<double> { double x0, x1; };
+//  * FP32 narrow layout (VX = 2): one pair c = (c0, c1) per row; the X sums
+//    are (L, R) + swap(c) with L, R shuffled straight into a register pair, so
+//    no pair is constructed (the 4-wide layout moves one half per X sum).
+template <typename T, int VX = Vec<T>::N> struct Rw;
+template <> struct Rw<float, 4> { float2 a, b; };
+template <> struct Rw<float, 2> { float2 a; };
+template <> struct Rw<double, 2> { double x0, x1; };
 
-__device__ __forceinline__ Rw<float> ld_row(const float* s) {
+__device__ __forceinline__ Rw<float, 4> ld_row(const float* s) {
     const float4 v = *reinterpret_cast<const float4*>(s);
-    return Rw<float>{make_float2(v.x, v.y), make_float2(v.z, v.w)};
+    return Rw<float, 4>{make_float2(v.x, v.y), make_float2(v.z, v.w)};
 }
 __device__ __forceinline__ Rw<double> ld_row(const double* s) {
     const double2 v = *reinterpret_cast<const double2*>(s);
     return Rw<double>{v.x, v.y};
 }
+template <int VX, typename T>
+__device__ __forceinline__ Rw<T, VX> ld_rowv(const T* s) {
+    if constexpr (sizeof(T) == 4 && VX == 2) return Rw<float, 2>{*reinterpret_cast<const float2*>(s)};
+    else return ld_row(s);
+}
+__device__ __forceinline__ void st_row(float* s, const Rw<float, 2>& r) { *reinterpret_cast<float2*>(s) = r.a; }
+#ifndef ST7_ST64
+#define ST7_ST64 0
+#endif
 __device__ __forceinline__ void st_row(float* s, const Rw<float>& r) {
+#if ST7_ST64   // two 8-byte stores: each packed pair is stored from its own register pair
+    reinterpret_cast<float2*>(s)[0] = r.a;
+    reinterpret_cast<float2*>(s)[1] = r.b;
+#else
     *reinterpret_cast<float4*>(s) = make_float4(r.a.x, r.a.y, r.b.x, r.b.y);
+#endif
 }
 __device__ __forceinline__ void st_row(double* s, const Rw<double>& r) {
     *reinterpret_cast<double2*>(s) = make_double2(r.x0, r.x1);
 }
 
-template <typename T, int VY> struct Bk { Rw<T> r[VY]; };
+template <typename T, int VY, int VX = Vec<T>::N> struct Bk { Rw<T, VX> r[VY]; };
 
 // Per-lane update coefficients.  A point on the x shell (x = 0 or nx-1) is
 // Dirichlet-fixed: it gets (alpha, beta) = (1, 0), so the update returns the
 // centre exactly (every neighbour sum is finite); y-shell rows are copied in a
 // warp-uniform branch, z-shell planes by the non-steady rounds.
-template <typename T> struct St7Coef;
-template <> struct St7Coef<float> {
+template <typename T, int VX = Vec<T>::N> struct St7Coef;
+template <> struct St7Coef<float, 2> {
+    float2 alA, beA;               // for the pair c = (c0, c1)
+    static __device__ __forceinline__ St7Coef make(float al, float be, uint32_t xfix) {
+        return St7Coef{make_float2(xfix & 1 ? 1.f : al, xfix & 2 ? 1.f : al),
+                       make_float2(xfix & 1 ? 0.f : be, xfix & 2 ? 0.f : be)};
+    }
+};
+template <> struct St7Coef<float, 4> {
     float2 alA, beA, alB, beB;     // for the pairs a = (c0, c1), b = (c2, c3)
     static __device__ __forceinline__ St7Coef make(float al, float be, uint32_t xfix) {  // xfix bit i: column i fixed
-#ifdef ST7_AB_SCALAR   // A/B timing only: ignores the x shell
-        xfix = xfix == 0xFu ? 0xFu : 0u;
+#ifdef ST7_AB_SCALAR   // A/B timing only: ignores the shell (wrong values there)
+        xfix = 0u;
 #endif
         St7Coef k;
         k.alA = make_float2(xfix & 1 ? 1.f : al, xfix & 2 ? 1.f : al);
@@ -117,7 +142,7 @@ template <> struct St7Coef<float> {
         return k;
     }
 };
-template <> struct St7Coef<double> {
+template <> struct St7Coef<double, 2> {
     double al0, be0, al1, be1;
     static __device__ __forceinline__ St7Coef make(double al, double be, uint32_t xfix) {
         return St7Coef{xfix & 1 ? 1.0 : al, xfix & 1 ? 0.0 : be, xfix & 2 ? 1.0 : al, xfix & 2 ? 0.0 : be};
@@ -125,8 +150,8 @@ template <> struct St7Coef<double> {
 };
 
 // y-shell rows (rowfix bit j) keep their value
-template <typename T, int VY>
-__device__ __forceinline__ void fix_rows(Bk<T, VY>& O, const Bk<T, VY>& H, uint32_t rowfix) {
+template <typename T, int VY, int VX>
+__device__ __forceinline__ void fix_rows(Bk<T, VY, VX>& O, const Bk<T, VY, VX>& H, uint32_t rowfix) {
 #pragma unroll
     for (int j = 0; j < VY; ++j)
         if (rowfix & (1u << j)) O.r[j] = H.r[j];
@@ -199,6 +224,43 @@ __device__ __forceinline__ void phaseA(const Bk<double, VY>& Zm, const Bk<double
     }
 }
 
+// narrow FP32 layout: one pair per row, X sums (L + c1, c0 + R) = (L, R) + swap(c)
+template <int NTX, int VY, bool EXACT>
+__device__ __forceinline__ void phaseA(const Bk<float, VY, 2>& Zm, const Bk<float, VY, 2>& H, const Rw<float, 2>& top,
+                                       const Rw<float, 2>& bot, const St7Coef<float, 2>& k, Bk<float, VY, 2>& A) {
+#pragma unroll
+    for (int j = 0; j < VY; ++j) {
+        const float2 LR = make_float2(__shfl_up_sync(0xffffffffu, H.r[j].a.y, 1, NTX),
+                                      __shfl_down_sync(0xffffffffu, H.r[j].a.x, 1, NTX));
+        const Rw<float, 2>& ym = j > 0 ? H.r[j - 1] : top;
+        const Rw<float, 2>& yp = j < VY - 1 ? H.r[j + 1] : bot;
+        const float2 c = H.r[j].a;
+        const float2 sx = __fadd2_rn(LR, make_float2(c.y, c.x));
+        const float2 sy = __fadd2_rn(ym.a, yp.a);
+        if (EXACT) {
+            A.r[j].a = __fadd2_rn(sx, sy);
+        } else {
+            const float2 s_ = __fadd2_rn(__fadd2_rn(sy, Zm.r[j].a), sx);
+            A.r[j].a = __ffma2_rn(k.alA, c, __fmul2_rn(k.beA, s_));
+        }
+    }
+}
+template <int VY, bool EXACT>
+__device__ __forceinline__ void phaseC(const Bk<float, VY, 2>& A, const Bk<float, VY, 2>& Zm, const Bk<float, VY, 2>& H,
+                                       const Bk<float, VY, 2>& F, const St7Coef<float, 2>& k, Bk<float, VY, 2>& O) {
+#pragma unroll
+    for (int j = 0; j < VY; ++j) {
+        if (EXACT) {
+            const float2 sa = __fadd2_rn(A.r[j].a, __fadd2_rn(Zm.r[j].a, F.r[j].a));
+            const float2 c = H.r[j].a;
+            O.r[j].a = make_float2(__fadd_rn(__fmul_rn(k.alA.x, c.x), __fmul_rn(k.beA.x, sa.x)),
+                                   __fadd_rn(__fmul_rn(k.alA.y, c.y), __fmul_rn(k.beA.y, sa.y)));
+        } else {
+            O.r[j].a = __ffma2_rn(k.beA, F.r[j].a, A.r[j].a);
+        }
+    }
+}
+
 // Phase C of one level: out = A + beta*F (fast), or the oracle's
 // alpha*c + beta*(q + (z- + z+)) with every operation rounded (exact)
 template <int VY, bool EXACT>
@@ -261,16 +323,20 @@ __device__ __forceinline__ St7Tile st7_tile(const St7Params& p, int tile, int D)
 // NT threads per CTA, MINB CTAs per SM (register cap 65536 / (NT * MINB));
 // SPLIT: two-phase rounds (false: level by level, the ablation ladder's
 // pre-ILP bar)
-template <typename T, int D, int NTX, int VY, bool EXACT, int NT, int MINB, bool SPLIT = true>
+// VXK: points per thread row (0: one 16-byte vector, 4 FP32 / 2 FP64; 2 for
+// FP32: the narrow layout, 32 threads across the 64-point tile row)
+template <typename T, int D, int NTX, int VY, bool EXACT, int NT, int MINB, bool SPLIT = true, int VXK = 0>
 __global__ void __launch_bounds__(NT, MINB)
 st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
-    constexpr int VX = sizeof(T) == 4 ? 4 : 2;
+    constexpr int VX = VXK ? VXK : (sizeof(T) == 4 ? 4 : 2);
     constexpr int TX = NTX * VX;
     const int NTH = blockDim.x;         // threads (<= NT): NTY rows of NTX threads
     const int NTY = NTH / NTX;
     const int TY = NTY * VY;
-    using V = typename std::conditional<sizeof(T) == 4, float4, double2>::type;
-    using B = Bk<T, VY>;
+    using V = typename std::conditional<VX * sizeof(T) == 16, typename std::conditional<sizeof(T) == 4, float4, double2>::type,
+                                        float2>::type;   // one exchanged row
+    using B = Bk<T, VY, VX>;
+    using RW = Rw<T, VX>;
 
     extern __shared__ __align__(128) unsigned char smem_raw[];
     const int tid = threadIdx.x;
@@ -312,7 +378,7 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
 #pragma unroll
         for (int k = 0; k < 3; ++k)
 #pragma unroll
-            for (int j = 0; j < VY; ++j) pl[l][k].r[j] = Rw<T>{};
+            for (int j = 0; j < VY; ++j) pl[l][k].r[j] = RW{};
 
     const int nzo = p.zb - p.za;
     int item = p.split[blockIdx.x];
@@ -369,7 +435,7 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
         const bool allfix = rowfix != 0 && (rowfix | rowout) == (1u << VY) - 1;
         const bool yslow = __any_sync(0xffffffffu, rowfix != 0 && !allfix);   // warp-uniform
         if (!(xg0 >= tl.ox0 && xg0 < tl.ox1)) rowmask = 0;    // vectors are all-in or all-out in x
-        const St7Coef<T> kc = St7Coef<T>::make(al, be, allfix ? 0xFu : xfix);
+        const St7Coef<T, VX> kc = St7Coef<T, VX>::make(al, be, allfix ? 0xFu : xfix);
 
         const int r0 = rl0, r1 = zb - 1 + D;
         // steady rounds: every level active, no z-shell plane among the computed ones
@@ -428,15 +494,15 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
             B acc[EXACT ? D + 1 : 1];
             auto level_A = [&](int l) {
                 const int k = l - 1;
-                Rw<T> top, bot;
+                RW top, bot;
                 if (l == 1) {   // level-0 neighbour rows of plane r-1 straight from the ring
                     const T* sl = ring + slot_m1 * slot_elems;
-                    top = ld_row(sl + top_off);
-                    bot = ld_row(sl + bot_off);
+                    top = ld_rowv<VX>(sl + top_off);
+                    bot = ld_rowv<VX>(sl + bot_off);
                 } else {        // rows the blocks above / below exchanged in round r-1
                     const V* xb = xbuf + ((l - 2) * 4 + (rpar ^ (l & 1)) * 2) * NTH;   // by level l-1 in round r-1
-                    top = ld_row(reinterpret_cast<const T*>(xb + NTH + tyu * NTX + tx));
-                    bot = ld_row(reinterpret_cast<const T*>(xb + tyd * NTX + tx));
+                    top = ld_rowv<VX>(reinterpret_cast<const T*>(xb + NTH + tyu * NTX + tx));
+                    bot = ld_rowv<VX>(reinterpret_cast<const T*>(xb + tyd * NTX + tx));
                 }
                 phaseA<NTX, VY, EXACT>(pl[k][PREV], pl[k][CUR], top, bot, kc, EXACT ? acc[EXACT ? l : 0] : pl[k][PREV]);
             };
@@ -446,7 +512,7 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                     mbar_wait(&bars[slot_r], par_r);
                     const T* s0 = ring + slot_r * slot_elems + my_off;
 #pragma unroll
-                    for (int j = 0; j < VY; ++j) pl[0][NEW].r[j] = ld_row(s0 + j * TX);
+                    for (int j = 0; j < VY; ++j) pl[0][NEW].r[j] = ld_rowv<VX>(s0 + j * TX);
                 }
             };
             // ---- phase C: the z+1 term along the level chain

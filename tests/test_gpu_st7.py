@@ -201,3 +201,30 @@ def test_degenerate_shapes_bitexact(oracle_lib, shape, dim_T):
     ref = oracle_lib.st7(a, 0.4, 0.1, T)
     got, _ = run_gpu(a, 0.4, 0.1, T, dim_T, exact=True)
     assert np.array_equal(got, ref)
+
+
+@pytest.mark.parametrize("variant", [4256, 2256, 214512, 214256, 1256, 94256, 22256, 2512, 4384])
+def test_kernel_variants_parity(oracle_lib, variant):
+    # every compiled 7-point kernel variant (ST_OPT_ST7_VARIANT): rows per thread, threads
+    # per CTA, CTAs per SM, the narrow FP32 layout (2 points per thread row) and the
+    # ablation-ladder kernels -- bit-exact (ladder kernels: tolerance build only) and
+    # within 1e-5 on ragged shapes at every depth the variant compiles
+    ladder = variant in (1256, 94256)
+    for k, (nx, ny, nz) in enumerate([(68, 52, 37), (200, 70, 11), (64, 130, 9)]):
+        a = stgen.grid7(nx, ny, nz, 300 + k, np.float32)
+        for D in (1, 2, 3, 4):
+            T = 2 * D + 1
+            ref = oracle_lib.st7(a, 0.4, 0.1, T)
+            for exact in ((False,) if ladder else (True, False)):
+                with st.Plan(nx, ny, nz, torch.float32, D) as p:
+                    p.set_bitexact(exact)
+                    p.set_option(st.ST_OPT_ST7_VARIANT, variant)
+                    x = torch.from_numpy(a).cuda()
+                    y = torch.empty_like(x)
+                    p.st7(x, y, 0.4, 0.1, T)
+                    p.sync()
+                    got = y.cpu().numpy()
+                if exact:
+                    assert np.array_equal(got, ref), (variant, nx, ny, nz, D)
+                else:
+                    assert relerr(got, ref) <= TOL[np.float32], (variant, nx, ny, nz, D)
