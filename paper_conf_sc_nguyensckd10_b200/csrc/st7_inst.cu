@@ -38,17 +38,17 @@ cudaError_t launch(const CUtensorMap* map, const St7Params& p, int grid, int thr
     return launch_pdl(p.pdl != 0, k, grid, threads, smem, s, *map, p);
 }
 
-template <int VY, int NT, int MINB = 1>
+template <int VY, int NT, int MINB = 1, int VX = 0>
 St7LaunchFn pick(int D) {
     switch (D) {
-        case 1: return launch<1, VY, NT, MINB>;
-        case 2: return launch<2, VY, NT, MINB>;
-        case 3: return launch<3, VY, NT, MINB>;
-        case 4: return launch<4, VY, NT, MINB>;
-        case 5: return launch<5, VY, NT, MINB>;
-        case 6: return launch<6, VY, NT, MINB>;
-        case 7: return launch<7, VY, NT, MINB>;
-        case 8: return launch<8, VY, NT, MINB>;
+        case 1: return launch<1, VY, NT, MINB, true, VX>;
+        case 2: return launch<2, VY, NT, MINB, true, VX>;
+        case 3: return launch<3, VY, NT, MINB, true, VX>;
+        case 4: return launch<4, VY, NT, MINB, true, VX>;
+        case 5: return launch<5, VY, NT, MINB, true, VX>;
+        case 6: return launch<6, VY, NT, MINB, true, VX>;
+        case 7: return launch<7, VY, NT, MINB, true, VX>;
+        case 8: return launch<8, VY, NT, MINB, true, VX>;
         default: return nullptr;
     }
 }
@@ -74,7 +74,8 @@ using namespace ST_UNIT_NS;
 St7LaunchFn ST_FN(int D, int VY, int NT, int MINB, int VX) {
     if constexpr (sizeof(TT) == 4) {
         if (VX == 2) {   // narrow FP32 layout: 32 threads x 2 points per tile row
-            if (MINB == 1 && VY == 4 && NT == 512) return pick4<4, 512, 1, true, 2>(D);
+            if (MINB == 1 && VY == 4 && NT == 512) return pick<4, 512, 1, 2>(D);
+            if (MINB == 1 && VY == 4 && NT == 384) return pick4<4, 384, 1, true, 2>(D);
             if (MINB == 1 && VY == 4 && NT == 256) return pick4<4, 256, 1, true, 2>(D);
             return nullptr;
         }
