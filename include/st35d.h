@@ -168,7 +168,9 @@ int st_plan_set_variant(st_plan* plan, int variant);
  *                       batched kernel (FP64 always batches).
  *   ST_OPT_LBM_KERNEL   0 (default) auto: dim_T = 1 push kernel when the plan's LBM
  *                       depth is 1, else the multi-level on-chip kernel; 1 push
- *                       (dim_T = 1 sweeps); 2 multi-level kernel at the plan depth.
+ *                       (dim_T = 1 sweeps); 2 multi-level kernel at the plan depth;
+ *                       3 gather form (collide pass, T-1 pull passes, stream pass;
+ *                       aligned stores; single domain).
  *   ST_OPT_OVERLAP      1 (default): Z-slab ghost exchange overlapped with the
  *                       interior sweep on a side stream; 0 serialised.
  *   ST_OPT_PDL          1 (default): 7-point sweeps chained with programmatic

@@ -398,7 +398,7 @@ extern "C" int st_plan_set_option(st_plan* p, int option, int value) {
             if (value < -1 || value > 1) return fail(ST_EINVAL, "ST_OPT_LBM_BATCHED %d", value);
             p->opt_lbm_batched = value; return ST_OK;
         case ST_OPT_LBM_KERNEL:
-            if (value < 0 || value > 2) return fail(ST_EINVAL, "ST_OPT_LBM_KERNEL %d", value);
+            if (value < 0 || value > 3) return fail(ST_EINVAL, "ST_OPT_LBM_KERNEL %d", value);
             p->opt_lbm_kernel = value; return ST_OK;
         case ST_OPT_OVERLAP: p->opt_overlap = value != 0; return ST_OK;
         case ST_OPT_PDL: p->opt_pdl = value != 0; return ST_OK;
@@ -1186,7 +1186,7 @@ static int max_lbm_depth(const st_plan* p) {
 }
 
 static bool lbm_use_push(const st_plan* p) {
-    if (p->opt_lbm_kernel == 1) return true;
+    if (p->opt_lbm_kernel == 1 || p->opt_lbm_kernel == 3) return true;
     if (p->opt_lbm_kernel == 2) return false;
     return max_lbm_depth(p) == 1;
 }
@@ -1273,6 +1273,34 @@ static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T
         }
         cudaError_t e = lbm_fl2(flags, p->fl2, p->nx, p->ny, p->dist.nzb, p->stream);
         if (e != cudaSuccess) return fail(ST_ECUDA, "fl2 prepass: %s", cudaGetErrorString(e));
+    }
+    if (p->opt_lbm_kernel == 3) {   // gather form: C, T-1 pulls, S (single domain)
+        if (p->dist.mode != Dist::SINGLE) return fail(ST_EUNSUPPORTED, "the gather-form LBM kernels are single-domain");
+        LbmParams prm{};
+        prm.nx = p->nx; prm.ny = p->ny; prm.nzb = p->nz; prm.zbase = 0; prm.nzg = p->nz;
+        prm.za = 0; prm.zb = p->nz;
+        prm.omega = omega;
+        if (p->dtype == ST_F32) lid_coeffs<float>(p->lid, prm.lidc);
+        else lid_coeffs<double>(p->lid, prm.lidc);
+        const long long cells = (long long)p->nx * p->ny * p->nz;
+        const int grid = (int)std::min<long long>((cells + 255) / 256, (long long)p->sms * 4);
+        const int dt = p->dtype == ST_F32 ? 0 : 1;
+        // T + 1 passes; C in place when T is odd so the result lands in f_dst
+        void* a = fsrc;
+        void* b = fdst;
+        auto pass = [&](int mode, void* from, void* to) -> int {
+            cudaError_t e = lbm_gather_launch(dt, p->exact, mode, from, to, p->fl2, prm, grid, p->stream);
+            if (e != cudaSuccess) return fail(ST_ECUDA, "lbm gather launch: %s", cudaGetErrorString(e));
+            ++p->launches;
+            return ST_OK;
+        };
+        if (T % 2) { rc = pass(LBM_COLLIDE, a, a); }
+        else { rc = pass(LBM_COLLIDE, a, b); std::swap(a, b); }
+        for (int t = 1; t < T && !rc; ++t) { rc = pass(LBM_PULL, a, b); std::swap(a, b); }
+        if (!rc) rc = pass(LBM_STREAM, a, b);
+        if (rc) return rc;
+        CUDA_TRY(cudaGetLastError());
+        return ST_OK;
     }
     std::vector<int> ds = push ? std::vector<int>(T, 1) : sweep_depths(T, max_lbm_depth(p));
     rc = run_sweeps(p, ds, fsrc, fdst, 19, flags, [&](const void* a, void* b, int d, const SlabView& sv) {

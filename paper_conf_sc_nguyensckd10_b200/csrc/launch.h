@@ -47,6 +47,8 @@ constexpr int ST13_MAX_DIM_T = 4;
 bool lbm_push_batched(int esize, int nx, int ny, int nzb, int force);   // kernel choice (also sets the grid)
 cudaError_t lbm_push_launch(int dtype, bool exact, bool slab, bool batched, const void* src, void* dst,
                             const uint8_t* fl2, const LbmParams& p, int grid, cudaStream_t s);
+cudaError_t lbm_gather_launch(int dtype, bool exact, int mode, const void* src, void* dst, const uint8_t* fl2,
+                              const LbmParams& p, int grid, cudaStream_t s);
 cudaError_t lbm35_launch(int dtype, bool exact, int D, const Lbm35Params& p, int grid, int threads, size_t smem,
                          cudaStream_t s);
 cudaError_t st7_naive_launch(int dtype, const void* in, void* out, int nx, int ny, int nz, double alpha,

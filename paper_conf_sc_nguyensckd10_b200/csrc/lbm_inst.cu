@@ -50,6 +50,26 @@ cudaError_t lbm_push_launch(int dtype, bool exact, bool slab, bool batched, cons
                  : push_s<double, false>(slab, batched, src, dst, fl2, p, grid, s);
 }
 
+template <typename T, bool E>
+static cudaError_t gather_t(int mode, const void* src, void* dst, const uint8_t* fl2, const LbmParams& p, int grid,
+                            cudaStream_t s) {
+    const T* a = static_cast<const T*>(src);
+    T* b = static_cast<T*>(dst);
+    if (mode == LBM_COLLIDE) lbm_gather_kernel<T, E, LBM_COLLIDE><<<grid, 256, 0, s>>>(a, b, fl2, p);
+    else if (mode == LBM_PULL) lbm_gather_kernel<T, E, LBM_PULL><<<grid, 256, 0, s>>>(a, b, fl2, p);
+    else lbm_gather_kernel<T, E, LBM_STREAM><<<grid, 256, 0, s>>>(a, b, fl2, p);
+    return cudaGetLastError();
+}
+
+// gather-form passes (mode LBM_COLLIDE / LBM_PULL / LBM_STREAM), single domain
+cudaError_t lbm_gather_launch(int dtype, bool exact, int mode, const void* src, void* dst, const uint8_t* fl2,
+                              const LbmParams& p, int grid, cudaStream_t s) {
+    if (dtype == 0) return exact ? gather_t<float, true>(mode, src, dst, fl2, p, grid, s)
+                                 : gather_t<float, false>(mode, src, dst, fl2, p, grid, s);
+    return exact ? gather_t<double, true>(mode, src, dst, fl2, p, grid, s)
+                 : gather_t<double, false>(mode, src, dst, fl2, p, grid, s);
+}
+
 template <typename T, int D, bool E>
 static cudaError_t l35_t(const Lbm35Params& p, int grid, int threads, size_t smem, cudaStream_t s) {
     auto k = lbm_35d_kernel<T, D, E>;

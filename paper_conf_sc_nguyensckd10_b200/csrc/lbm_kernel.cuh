@@ -245,6 +245,66 @@ lbm_push_kernel(const T* __restrict__ src, T* __restrict__ dst, const uint8_t* _
     }
 }
 
+
+// ---------------------------------------------------------------------------
+// Gather form (a10: every store of a cell's 19 values is aligned and
+// coalesced at the cell itself, no x-shifted scatter).  With P = S.C the push
+// step (collide, then stream), T push steps are  P^T = S . (C.S)^(T-1) . C:
+// one collide-only pass, T-1 pull passes (gather the neighbours'
+// post-collision values, then collide) and one stream-only pass.  The stored
+// intermediate state is post-collision; every (cell, population) sees the
+// same operations as in the push kernel, so the result is bit-identical.
+// Bounce-back in gather form: the value arriving at x in direction i comes
+// from x - e_i; if that cell is WALL it is x's own post-collision value of
+// opp(i) (the half-way reflection), if LID the same minus (6 w e.u)_opp(i).
+// fl2 marks FLUID cells with a non-FLUID neighbour; only they read flags.
+// ---------------------------------------------------------------------------
+enum { LBM_COLLIDE = 0, LBM_PULL = 1, LBM_STREAM = 2 };
+
+template <typename T, bool E, int MODE>
+__global__ void __launch_bounds__(256, 4)
+lbm_gather_kernel(const T* src, T* dst, const uint8_t* __restrict__ fl2, const LbmParams p) {
+    // (src may equal dst for the in-place collide pass: no __restrict__ on the lattices)
+    const size_t plane = (size_t)p.nx * p.ny;
+    const long long nc = (long long)(plane * p.nzb);
+    const size_t c0 = (size_t)p.za * plane;
+    const size_t ncell = (size_t)(p.zb - p.za) * plane;
+    const T omega = T(p.omega);
+    for (size_t t = blockIdx.x * (size_t)blockDim.x + threadIdx.x; t < ncell; t += (size_t)gridDim.x * blockDim.x) {
+        const size_t c = c0 + t;
+        const uint32_t fl = fl2[c];
+        const T* s = src + c;
+        T* d = dst + c;
+        T f[19];
+        if ((fl & 0x7fu) != 0 || MODE == LBM_COLLIDE) {
+#pragma unroll
+            for (int i = 0; i < 19; ++i) f[i] = s[(long long)i * nc];
+            if ((fl & 0x7fu) == 0) collide<T, E>(f, omega);   // COLLIDE on a FLUID cell
+#pragma unroll
+            for (int i = 0; i < 19; ++i) d[(long long)i * nc] = f[i];
+            continue;
+        }
+        auto gather = [&](auto Ic) {
+            constexpr int I = decltype(Ic)::value;
+            const long long off = (long long)D3Q19<I>::ex + (long long)D3Q19<I>::ey * p.nx +
+                                  (long long)D3Q19<I>::ez * (long long)plane;
+            if constexpr (I == 0) {
+                f[0] = s[0];
+            } else {
+                const uint32_t sf = (fl & 0x80u) ? (uint32_t)__ldg(fl2 + (long long)c - off) & 0x7fu : 0u;
+                if (sf == 0) f[I] = s[(long long)I * nc - off];
+                else if (sf == 1) f[I] = s[(long long)D3Q19<I>::opp * nc];
+                else f[I] = Ar<T, E>::sub(s[(long long)D3Q19<I>::opp * nc], T(p.lidc[D3Q19<I>::opp]));
+            }
+        };
+        [&]<int... Is>(std::integer_sequence<int, Is...>) { (gather(std::integral_constant<int, Is>{}), ...); }
+        (std::make_integer_sequence<int, 19>{});
+        if (MODE == LBM_PULL) collide<T, E>(f, omega);
+#pragma unroll
+        for (int i = 0; i < 19; ++i) d[(long long)i * nc] = f[i];
+    }
+}
+
 // ---------------------------------------------------------------------------
 // lbm_35d_kernel: the 3.5D-blocked D3Q19 sweep (dim_T = D levels on chip).
 //

@@ -229,3 +229,29 @@ def test_batched_kernel_above_2_24_cells(oracle_lib):
     ref = oracle_lib.lbm(f0, flags, 1.6, T)
     assert np.array_equal(run_gpu(f0, flags, 1.6, T, exact=True), ref)
     assert relerr(run_gpu(f0, flags, 1.6, T), ref) <= TOL[np.float32]
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+@pytest.mark.parametrize("T", [1, 2, 5])
+def test_gather_form_kernels(oracle_lib, dtype, T):
+    # ST_OPT_LBM_KERNEL 3: collide pass, T-1 pull (gather) passes, stream pass with
+    # aligned stores -- the same operations per (cell, population) as the push step,
+    # so bit-identical to the oracle, interior obstacle included
+    nx, ny, nz = 96, 50, 13
+    flags = stgen.cavity_flags(nx, ny, nz)
+    flags[nz // 2, 5:8, 7:12] = stgen.WALL
+    f0 = stgen.lbm_random(nx, ny, nz, 3, dtype)
+    ref = oracle_lib.lbm(f0, flags, 1.6, T)
+    for exact in (True, False):
+        with st.Plan(nx, ny, nz, torch.float32 if dtype == np.float32 else torch.float64, 1) as p:
+            p.set_bitexact(exact)
+            p.set_option(st.ST_OPT_LBM_KERNEL, 3)
+            a = torch.from_numpy(f0).cuda()
+            b = torch.empty_like(a)
+            p.lbm(a, b, 1.6, T, torch.from_numpy(flags).cuda())
+            p.sync()
+            got = b.cpu().numpy()
+        if exact:
+            assert np.array_equal(got, ref)
+        else:
+            assert relerr(got, ref) <= TOL[dtype]
