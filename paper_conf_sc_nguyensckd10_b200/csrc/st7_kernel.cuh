@@ -477,16 +477,19 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
             }
             // Non-steady rounds (prolog, epilog, z-shell planes, warps with an
             // unaligned y-shell row) run the same body plus checks: a level whose
-            // plane lies outside its range computes a finite value nobody reads;
-            // a level on a z-shell plane copies its centre (fixed boundary); the
-            // final level stores only output planes.
-            bool zf[D + 1];
+            // plane lies outside its range is skipped (warp-uniform); a level on a
+            // z-shell plane copies its centre (fixed boundary); the final level
+            // stores only output planes.
+            bool zf[D + 1], act[D + 1];
 #pragma unroll
             for (int l = 1; l <= D; ++l) {
                 zf[l] = false;
-                if (!STEADY) {
+                act[l] = true;
+                if (!STEADY) {   // level l computes plane r - l: inside its range, or skipped
                     const int zg = p.zbase + r - l;
                     zf[l] = zg == 0 || zg == p.nzg - 1;
+                    const int lo = max(za - (D - l), zmin), hi = min(zb - 1 + (D - l), zmax);
+                    act[l] = r - l >= lo && r - l <= hi;
                 }
             }
             // ---- phase A: in-plane part of every level (no dependence on this round's planes);
@@ -535,16 +538,21 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                         if (rowmask & (1u << j)) st_row(pout + j * p.nx, out.r[j]);
                 }
             };
+            // (a skipped level's planes are never read: the level above is outside
+            // its range in the rounds that would read them)
             if (SPLIT) {   // all in-plane parts first, then the z+1 chain
 #pragma unroll
-                for (int l = 1; l <= D; ++l) level_A(l);
+                for (int l = 1; l <= D; ++l)
+                    if (act[l]) level_A(l);
                 load0();
 #pragma unroll
-                for (int l = 1; l <= D; ++l) level_C(l);
+                for (int l = 1; l <= D; ++l)
+                    if (act[l]) level_C(l);
             } else {           // level by level
                 load0();
 #pragma unroll
-                for (int l = 1; l <= D; ++l) { level_A(l); level_C(l); }
+                for (int l = 1; l <= D; ++l)
+                    if (act[l]) { level_A(l); level_C(l); }
             }
             __syncthreads();
             pout += plane;
