@@ -519,9 +519,20 @@ static bool overlap(const void* a, const void* b, size_t n) {
 // over a greedy cut.
 static void split_work(int ntiles, int nzo, int d, int G, int* split, int zchunk = 0) {
     const long long work = (long long)ntiles * nzo;
-    // measured on B200 (ST_SPLIT_OVH A/B, 256^3): 4 plane-equivalents per segment is
-    // best at dim_T 3 and 4 (+2 % over the d + 2 model); shallower sweeps restart cheaper
-    const long long ovh = std::min(d + 1, 4);
+    // per-segment restart cost in plane-equivalents: the 2d prolog rounds of a
+    // segment (levels start one after another, no output) plus segment set-up
+    // and first-load latency.  Measured on B200: per-CTA globaltimer trace
+    // (tools/trace7.py, 256^3 FP32 d = 4): prolog 5.9 us (compile-time prolog
+    // rounds; 9.8 us with checked rounds) vs 0.93 us per steady plane; A/B of
+    // the constant (256^3 FP32, Gupd/s): d = 4: 4 -> 1275, 7 -> 1319,
+    // 8 -> 1368, 9 -> 1405, 10 -> 1326; d = 3: 4 -> 1231, 7 -> 1256,
+    // 8 -> 1308, 9 -> 1295; d = 2: 4 -> 1062, 6 -> 1151.  The spread beyond
+    // the model comes from which CTAs get a second segment.
+#ifdef ST_SPLIT_OVH_AB
+    const long long ovh = ST_SPLIT_OVH_AB;   // A/B tuning builds only
+#else
+    const long long ovh = std::min(2LL * d + 2, 9LL);
+#endif
     auto cuts = [&](long long C, int* out) {   // CTAs needed with per-CTA cost cap C
         if (C <= ovh) return G + 1;             // no CTA could take a plane
         long long it = 0;

@@ -95,4 +95,16 @@ St7LaunchFn ST_FN(int D, int VY, int NT, int MINB, int VX) {
     return nullptr;
 }
 
+#if defined(ST7_TRACE) && !ST_EXACT
+extern "C" int ST_CAT(st7_trace_read_, ST_TNAME)(void* host) {   // A/B diagnostics build only
+    return (int)cudaMemcpyFromSymbol(host, st7_trace_buf, sizeof(st7_trace_buf));
+}
+extern "C" int ST_CAT(st7_trace_rounds_, ST_TNAME)(void* host) {
+    return (int)cudaMemcpyFromSymbol(host, st7_trace_rnd, sizeof(st7_trace_rnd));
+}
+extern "C" int ST_CAT(st7_trace_issue_, ST_TNAME)(void* host) {
+    return (int)cudaMemcpyFromSymbol(host, st7_trace_iss, sizeof(st7_trace_iss));
+}
+#endif
+
 }  // namespace st35d

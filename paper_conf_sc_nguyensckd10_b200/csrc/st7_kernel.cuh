@@ -325,6 +325,33 @@ __device__ __forceinline__ St7Tile st7_tile(const St7Params& p, int tile, int D)
 // pre-ILP bar)
 // VXK: points per thread row (0: one 16-byte vector, 4 FP32 / 2 FP64; 2 for
 // FP32: the narrow layout, 32 threads across the 64-point tile row)
+// compile-time loop: f(integral_constant<int, I>) for I = B..E-1
+template <int B, int E, typename F>
+__device__ __forceinline__ void static_for(F&& f) {
+    if constexpr (B < E) {
+        f(std::integral_constant<int, B>{});
+        static_for<B + 1, E>(f);
+    }
+}
+
+#ifdef ST7_TRACE
+// A/B diagnostics build only (-DST7_TRACE): per CTA globaltimer stamps
+// [entry, after pdl_wait, (segment start, first steady round, steady end) x 3,
+// end, segment count, first 3 segment lengths (16 bits each)]
+static __device__ unsigned long long st7_trace_buf[ST7_MAX_GRID][16];
+// first 16 rounds of segment 0: [round][0] plane landed (after mbar_wait), [1] round end
+static __device__ unsigned long long st7_trace_rnd[ST7_MAX_GRID][16][2];
+static __device__ unsigned long long st7_trace_iss[ST7_MAX_GRID][16];   // segment 0: issue time of load k
+__device__ __forceinline__ unsigned long long st7_gtime() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+#define ST7_STAMP(i, v) do { if (threadIdx.x == 0) st7_trace_buf[blockIdx.x][i] = (v); } while (0)
+#else
+#define ST7_STAMP(i, v) do { } while (0)
+#endif
+
 template <typename T, int D, int NTX, int VY, bool EXACT, int NT, int MINB, bool SPLIT = true, int VXK = 0>
 __global__ void __launch_bounds__(NT, MINB)
 st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
@@ -339,6 +366,10 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
     using RW = Rw<T, VX>;
 
     extern __shared__ __align__(128) unsigned char smem_raw[];
+#ifdef ST7_TRACE
+    ST7_STAMP(0, st7_gtime());
+    int nseg_tr = 0;
+#endif
     const int tid = threadIdx.x;
     const int tx = tid % NTX;
     const int ty = tid / NTX;
@@ -369,6 +400,9 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
     // (this sweep's input) and its reads of our output buffer are complete here
     pdl_trigger();
     pdl_wait();
+#ifdef ST7_TRACE
+    ST7_STAMP(1, st7_gtime());
+#endif
 
     // register window: pl[k][*] holds planes of level k (0..D-1), three slots
     // rotating with the round (z-1, z, new); level 0 is loaded from the ring
@@ -410,6 +444,12 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
 
     while (item < item_end) {
         const Seg sg = seg_at(item);
+#ifdef ST7_TRACE
+        if (nseg_tr < 3) ST7_STAMP(2 + 3 * nseg_tr, st7_gtime());
+        if (nseg_tr < 3) ST7_STAMP(14, (nseg_tr ? st7_trace_buf[blockIdx.x][14] : 0ull) |
+                                           ((unsigned long long)(sg.zb - sg.za) << (16 * nseg_tr)));
+        ++nseg_tr;
+#endif
         const int za = sg.za, zb = sg.zb, rl0 = sg.rl0, rl1 = sg.rl1;
         item += zb - za;
         const bool has_next = item < item_end;
@@ -449,6 +489,9 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                 const uint32_t k = (kbase + (q - rl0)) % RING;
                 mbar_arrive_expect_tx(&bars[k], slot_bytes);
                 tma_load_3d(ring + k * slot_elems, &tmap, &bars[k], tl.Lx, tl.Ly, q);
+#ifdef ST7_TRACE
+                if (nseg_tr == 1 && q - rl0 < 16) st7_trace_iss[blockIdx.x][q - rl0] = st7_gtime();
+#endif
             }
             pre = 0;
         }
@@ -458,9 +501,12 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
         uint32_t slot_f = (kbase + PF) % RING;
         uint32_t slot_m1 = (slot_r + RING - 1) % RING;
 
-        auto round = [&](auto PHc, auto STEADYc, int r) {
+        // NACTc: -1 = checked round; n >= 0 = unchecked round with levels 1..n
+        // active (n = D: a steady round; n < D: a prolog round, no output)
+        auto round = [&](auto PHc, auto NACTc, int r) {
             constexpr int PH = decltype(PHc)::value;
-            constexpr bool STEADY = decltype(STEADYc)::value;
+            constexpr int NACT = decltype(NACTc)::value;
+            constexpr bool STEADY = NACT >= 0;
             constexpr int PREV = PH % 3, CUR = (PH + 1) % 3, NEW = (PH + 2) % 3;
             const int rpar = r & 1;
             // load plane r + PF into the slot plane r-2 left (free since round r-1's barrier)
@@ -468,6 +514,9 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                 if (r + PF <= rl1) {
                     mbar_arrive_expect_tx(&bars[slot_f], slot_bytes);
                     tma_load_3d(ring + slot_f * slot_elems, &tmap, &bars[slot_f], tl.Lx, tl.Ly, r + PF);
+#ifdef ST7_TRACE
+                    if (nseg_tr == 1 && r + PF - rl0 < 16) st7_trace_iss[blockIdx.x][r + PF - rl0] = st7_gtime();
+#endif
                 } else if (has_next && pre < PF && pre == r + PF - rl1 - 1 && nx.rl0 + pre <= nx.rl1) {
                     // sequence kbase + (r + PF - rl0) is the next segment's plane rl0' + pre
                     mbar_arrive_expect_tx(&bars[slot_f], slot_bytes);
@@ -484,7 +533,7 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
 #pragma unroll
             for (int l = 1; l <= D; ++l) {
                 zf[l] = false;
-                act[l] = true;
+                act[l] = !STEADY || l <= NACT;
                 if (!STEADY) {   // level l computes plane r - l: inside its range, or skipped
                     const int zg = p.zbase + r - l;
                     zf[l] = zg == 0 || zg == p.nzg - 1;
@@ -513,6 +562,9 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
             auto load0 = [&]() {
                 if (STEADY || r <= rl1) {
                     mbar_wait(&bars[slot_r], par_r);
+#ifdef ST7_TRACE
+                    if (tid == 0 && nseg_tr == 1 && r - r0 < 16) st7_trace_rnd[blockIdx.x][r - r0][0] = st7_gtime();
+#endif
                     const T* s0 = ring + slot_r * slot_elems + my_off;
 #pragma unroll
                     for (int j = 0; j < VY; ++j) pl[0][NEW].r[j] = ld_rowv<VX>(s0 + j * TX);
@@ -555,6 +607,9 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
                     if (act[l]) { level_A(l); level_C(l); }
             }
             __syncthreads();
+#ifdef ST7_TRACE
+            if (tid == 0 && nseg_tr == 1 && r - r0 < 16) st7_trace_rnd[blockIdx.x][r - r0][1] = st7_gtime();
+#endif
             pout += plane;
             slot_m1 = slot_r;
             if (++slot_r == (uint32_t)RING) { slot_r = 0; par_r ^= 1; }
@@ -563,29 +618,54 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
         using I0 = std::integral_constant<int, 0>;
         using I1 = std::integral_constant<int, 1>;
         using I2 = std::integral_constant<int, 2>;
+        using ND = std::integral_constant<int, D>;
+        using NCHK = std::integral_constant<int, -1>;
         // Steady rounds (every level active, no z-shell plane, no unaligned
         // y-shell row in the warp) run as
         // back-to-back phase triples without any check; the other rounds take
         // the checked body.  ph = (r - r0) mod 3 selects the register slots.
         const int rs1x = rs1;
         int r = r0, ph = 0;
+        // prolog of a segment away from the z faces: round k = 0..2D-1 runs
+        // levels 1..k/2 (level l starts at plane za - D + l in round 2l) as
+        // compile-time rounds without checks; its register phase starts at
+        // (-2D) mod 3 so that the steady triples follow at phase 0
+        if (!yslow && r0 == za - D && r0 + 2 * D == rs0 && p.zbase + za - D >= 1 &&
+            p.zbase + za + D < p.nzg - 1 && za + D - 1 <= rl1) {
+            constexpr int PH0 = (3 - (2 * D) % 3) % 3;
+            static_for<0, 2 * D>([&](auto K) {
+                constexpr int k = decltype(K)::value;
+                round(std::integral_constant<int, (PH0 + k) % 3>{}, std::integral_constant<int, k / 2>{}, r0 + k);
+            });
+            r = r0 + 2 * D;
+        }
         while (r <= r1) {
             if (ph == 0 && !yslow && r >= rs0 && r + 2 <= rs1x) {
+#ifdef ST7_TRACE
+                if (nseg_tr <= 3) ST7_STAMP(3 * nseg_tr, st7_gtime());
+#endif
                 do {
-                    round(I0{}, std::true_type{}, r);
-                    round(I1{}, std::true_type{}, r + 1);
-                    round(I2{}, std::true_type{}, r + 2);
+                    round(I0{}, ND{}, r);
+                    round(I1{}, ND{}, r + 1);
+                    round(I2{}, ND{}, r + 2);
                     r += 3;
                 } while (r + 2 <= rs1x);
+#ifdef ST7_TRACE
+                if (nseg_tr <= 3) ST7_STAMP(3 * nseg_tr + 1, st7_gtime());
+#endif
                 continue;
             }
-            if (ph == 0) round(I0{}, std::false_type{}, r);
-            else if (ph == 1) round(I1{}, std::false_type{}, r);
-            else round(I2{}, std::false_type{}, r);
+            if (ph == 0) round(I0{}, NCHK{}, r);
+            else if (ph == 1) round(I1{}, NCHK{}, r);
+            else round(I2{}, NCHK{}, r);
             ++r;
             ph = ph == 2 ? 0 : ph + 1;
         }
     }
+#ifdef ST7_TRACE
+    ST7_STAMP(12, st7_gtime());
+    ST7_STAMP(13, (unsigned long long)nseg_tr);
+#endif
 }
 
 }  // namespace st35d
