@@ -499,7 +499,8 @@ def main():
                                             "roofline": {"bound": "hbm", "achieved": round(gbs, 1),
                                                          "peak": hbm_gbs, "unit": "GB/s",
                                                          "frac": round(gbs / hbm_gbs, 4)},
-                                            "launches": pl.last_launches()}
+                                            "launches": pl.last_launches(),
+                                            "kernel": pl.info(True)["kernel"]}
             del fa, fb, f0, flags
         # configs[4] lattice on one GPU (1024^3 FP32 cavity from rest: the strong-scaling base,
         # 163 GB for the two lattices), built on the device
@@ -528,6 +529,7 @@ def main():
                 gbs = LBM_BYTES[4] * cells * Tb / (msl / 1e3) / 1e9
                 extras["lbm_f32_1024"] = {"value": round(cells * Tb / (msl / 1e3) / 1e6, 1), "unit": "MLUPS",
                                           "dim_T": 1, "T": Tb, "ms_per_step": round(msl, 3),
+                                          "kernel": pl.info(True)["kernel"],
                                           "note": "configs[4] lattice on one GPU (strong-scaling base)",
                                           "roofline": {"bound": "hbm", "achieved": round(gbs, 1), "peak": hbm_gbs,
                                                        "unit": "GB/s", "frac": round(gbs / hbm_gbs, 4)}}

@@ -166,11 +166,17 @@ int st_plan_set_variant(st_plan* plan, int variant);
  *   ST_OPT_LBM_BATCHED  -1 (default) auto: FP32 lattices above 2^24 cells use the
  *                       batched-flag push kernel; 0 / 1 force the per-direction /
  *                       batched kernel (FP64 always batches).
- *   ST_OPT_LBM_KERNEL   0 (default) auto: dim_T = 1 push kernel when the plan's LBM
- *                       depth is 1, else the multi-level on-chip kernel; 1 push
+ *   ST_OPT_LBM_KERNEL   0 (default) auto: when the plan's LBM depth is 1, the
+ *                       TMA gather form (4) for FP32 single-domain runs of T >= 4
+ *                       with nx * 4 % 16 == 0, else the dim_T = 1 push kernel; at
+ *                       depth >= 2 the multi-level on-chip kernel; 1 push
  *                       (dim_T = 1 sweeps); 2 multi-level kernel at the plan depth;
  *                       3 gather form (collide pass, T-1 pull passes, stream pass;
- *                       aligned stores; single domain).
+ *                       aligned stores; single domain); 4 the same with the
+ *                       pull passes fed by TMA (4D boxes shifted per population,
+ *                       S-stage shared-memory ring; needs nx * sizeof(T) % 16 == 0,
+ *                       else the plain pull kernel runs).
+ *   ST_OPT_LBM_STAGES   0 (default) auto; 1..8 stages of the TMA pull ring.
  *   ST_OPT_OVERLAP      1 (default): Z-slab ghost exchange overlapped with the
  *                       interior sweep on a side stream; 0 serialised.
  *   ST_OPT_PDL          1 (default): 7-point sweeps chained with programmatic
@@ -186,7 +192,7 @@ int st_plan_set_variant(st_plan* plan, int variant);
  *                       PAPER.md P:275-281).
  * Results do not depend on any option.  Unknown option or value: ST_EINVAL. */
 enum { ST_OPT_LBM_BATCHED = 1, ST_OPT_LBM_KERNEL = 2, ST_OPT_OVERLAP = 3, ST_OPT_PDL = 4, ST_OPT_ST7_VARIANT = 5,
-       ST_OPT_ZCHUNK = 6 };
+       ST_OPT_ZCHUNK = 6, ST_OPT_LBM_STAGES = 7 };
 int st_plan_set_option(st_plan* plan, int option, int value);
 
 /* st_plan_autotune_report — choose the 7-point sweep depth (the paper's
@@ -295,7 +301,9 @@ typedef struct {
     int threads;            /* threads per CTA                                  */
     int smem_bytes;         /* dynamic shared memory per CTA                    */
     double kappa;           /* eq. (2) analog: computed / useful points         */
-    int kernel;             /* internal variant id                               */
+    int kernel;             /* internal variant id; LBM (after a run: the kernel
+                               it used): 100 push, 200+d multi-level of depth d,
+                               300 gather form, 400 gather form with TMA pulls  */
     int dim_t_sweep;        /* deepest sweep actually run (<= dim_T, see above)  */
     int ring;               /* TMA plane-ring slots (ring-2 planes in flight)    */
 } st_plan_info;

@@ -22,6 +22,7 @@ ST_OK, ST_EINVAL, ST_ENOMEM, ST_ECUDA, ST_ENCCL, ST_EUNSUPPORTED = 0, -1, -2, -3
 ST_FLUID, ST_WALL, ST_LID = 0, 1, 2
 ST_MAX_DIM_T = 8
 ST_OPT_LBM_BATCHED, ST_OPT_LBM_KERNEL, ST_OPT_OVERLAP, ST_OPT_PDL, ST_OPT_ST7_VARIANT, ST_OPT_ZCHUNK = 1, 2, 3, 4, 5, 6
+ST_OPT_LBM_STAGES = 7
 _ERRNAMES = {-1: "ST_EINVAL", -2: "ST_ENOMEM", -3: "ST_ECUDA", -4: "ST_ENCCL", -5: "ST_EUNSUPPORTED"}
 
 

@@ -47,6 +47,7 @@ COMMON = ARCH + ["-O3", "-lineinfo", "-std=c++20", "--expt-relaxed-constexpr", "
 UNITS = [
     ("api.cu", "api.o", []),
     ("lbm_inst.cu", "lbm_inst.o", []),
+    ("lbm_tma.cu", "lbm_tma.o", []),
     ("naive.cu", "naive.o", []),
     ("st27.cu", "st27.o", []),
     ("st13_inst.cu", "st13_inst.o", []),
@@ -62,17 +63,28 @@ def _deps():
     return sorted(glob.glob(os.path.join(CSRC, "*")) + glob.glob(os.path.join(ROOT, "include", "*.h")))
 
 
+def _unit_deps(obj: str) -> list[str]:
+    """headers the object was compiled from (nvcc -MD), else every source file"""
+    dep = obj + ".d"
+    if not os.path.exists(dep):
+        return _deps()
+    txt = open(dep).read().replace("\\\n", " ")
+    files = [f for f in txt.split(":", 1)[-1].split() if f.startswith(ROOT)]
+    return files + [os.path.abspath(__file__)] if files else _deps()
+
+
 def _stale(obj: str, src: str) -> bool:
     if not os.path.exists(obj):
         return True
     t = os.path.getmtime(obj)
-    return any(os.path.getmtime(d) > t for d in _deps())
+    return any(not os.path.exists(d) or os.path.getmtime(d) > t for d in _unit_deps(obj))
 
 
 def _compile(src, obj, extra, verbose):
-    cmd = [NVCC, *COMMON, *extra, "-c", os.path.join(CSRC, src), "-o", obj]
+    md = ["-MD", "-MF", obj + ".d"]
+    cmd = [NVCC, *COMMON, *extra, *md, "-c", os.path.join(CSRC, src), "-o", obj]
     if src.endswith(".cpp"):
-        cmd = [NVCC, *COMMON, *extra, "-x", "cu", "-c", os.path.join(CSRC, src), "-o", obj]
+        cmd = [NVCC, *COMMON, *extra, *md, "-x", "cu", "-c", os.path.join(CSRC, src), "-o", obj]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
         cmd.insert(1, "-Xptxas=-warn-spills")

@@ -79,6 +79,12 @@ static int encode_3d(CUtensorMap* map, const void* base, st_dtype dt, int nx, in
     return ST_OK;
 }
 
+// SoA D3Q19 lattice as one 3D map (x, y, 19 nz): population i is planes [i nz, i nz + nz)
+static int encode_lbm(CUtensorMap* map, const void* base, st_dtype dt, int nx, int ny, int nz, int bx, int by) {
+    if (19LL * nz > (1LL << 31) - 1) return fail(ST_EUNSUPPORTED, "19 nz exceeds a TMA coordinate");
+    return encode_3d(map, base, dt, nx, ny, 19 * nz, bx, by);
+}
+
 // ----------------------------------------------------------------------------
 // plan
 // ----------------------------------------------------------------------------
@@ -112,7 +118,9 @@ struct st_plan {
     int launches = 0;
     // st_plan_set_option (include/st35d.h): tuning / test selections, no environment variables
     int opt_lbm_batched = -1;   // -1 auto
-    int opt_lbm_kernel = 0;     // 0 auto, 1 push, 2 multi-level
+    int opt_lbm_kernel = 0;     // 0 auto, 1 push, 2 multi-level, 3 gather form, 4 gather form + TMA pulls
+    int opt_lbm_stages = 0;     // TMA pull ring depth (0 auto)
+    int last_lbm_kernel = 0;    // kernel code of the last lbm_d3q19_run (st_plan_get_info)
     int opt_overlap = 1;
     int opt_pdl = 1;
     int opt_st7_variant = 0;    // 0 auto, else VY * 1000 + threads per CTA (+ 10000 * CTAs per SM)
@@ -398,8 +406,11 @@ extern "C" int st_plan_set_option(st_plan* p, int option, int value) {
             if (value < -1 || value > 1) return fail(ST_EINVAL, "ST_OPT_LBM_BATCHED %d", value);
             p->opt_lbm_batched = value; return ST_OK;
         case ST_OPT_LBM_KERNEL:
-            if (value < 0 || value > 3) return fail(ST_EINVAL, "ST_OPT_LBM_KERNEL %d", value);
+            if (value < 0 || value > 4) return fail(ST_EINVAL, "ST_OPT_LBM_KERNEL %d", value);
             p->opt_lbm_kernel = value; return ST_OK;
+        case ST_OPT_LBM_STAGES:
+            if (value < 0 || value > 8) return fail(ST_EINVAL, "ST_OPT_LBM_STAGES %d", value);
+            p->opt_lbm_stages = value; return ST_OK;
         case ST_OPT_OVERLAP: p->opt_overlap = value != 0; return ST_OK;
         case ST_OPT_PDL: p->opt_pdl = value != 0; return ST_OK;
         case ST_OPT_ZCHUNK:
@@ -454,7 +465,7 @@ extern "C" int st_plan_get_info(const st_plan* p, int lbm, st_plan_info* info) {
         info->tiles_x = g.tiles_x; info->tiles_y = g.tiles_y; info->ctas = p->sms; info->threads = 32 * g.TY;
         info->smem_bytes = (int)g.smem;
         info->kappa = (double)g.tiles_x * 32 * g.tiles_y * g.TY / ((double)p->nx * p->ny);
-        info->kernel = lbm_use_push(p) ? 100 : 200 + d;
+        info->kernel = p->last_lbm_kernel ? p->last_lbm_kernel : (lbm_use_push(p) ? 100 : 200 + d);
         info->dim_t_sweep = d;
         return ST_OK;
     }
@@ -1285,7 +1296,14 @@ static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T
         cudaError_t e = lbm_fl2(flags, p->fl2, p->nx, p->ny, p->dist.nzb, p->stream);
         if (e != cudaSuccess) return fail(ST_ECUDA, "fl2 prepass: %s", cudaGetErrorString(e));
     }
-    if (p->opt_lbm_kernel == 3) {   // gather form: C, T-1 pulls, S (single domain)
+    // FP32 single-domain dim_T = 1 runs of T >= 4 steps: the gather form with TMA-fed
+    // pull passes (measured on B200, 256^3 cavity: 33.1 vs 25.8 GLUPS for the push
+    // kernel; FP64 keeps push, 18.4 vs 16.7).  T + 1 passes.
+    int gk = p->opt_lbm_kernel;
+    if (gk == 0 && push && p->dist.mode == Dist::SINGLE && p->dtype == ST_F32 && T >= 4 &&
+        ((size_t)p->nx * esize(p->dtype)) % 16 == 0)
+        gk = 4;
+    if (gk == 3 || gk == 4) {   // gather form: C, T-1 pulls, S (single domain)
         if (p->dist.mode != Dist::SINGLE) return fail(ST_EUNSUPPORTED, "the gather-form LBM kernels are single-domain");
         LbmParams prm{};
         prm.nx = p->nx; prm.ny = p->ny; prm.nzb = p->nz; prm.zbase = 0; prm.nzg = p->nz;
@@ -1296,11 +1314,41 @@ static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T
         const long long cells = (long long)p->nx * p->ny * p->nz;
         const int grid = (int)std::min<long long>((cells + 255) / 256, (long long)p->sms * 4);
         const int dt = p->dtype == ST_F32 ? 0 : 1;
+        // TMA pulls (a10): 4D maps of both lattices, S-stage ring, CTAs per SM from shared memory
+        const bool tma = gk == 4 && ((size_t)p->nx * esize(p->dtype)) % 16 == 0;
+        p->last_lbm_kernel = tma ? 400 : 300;
+        CUtensorMap map_src[2], map_dst[2];
+        int tgrid = 0, stages = 0;
+        if (tma) {
+            int bx, by, halo;
+            lbm_pull_tma_box(dt, &bx, &by, &halo);
+            for (int w = 0; w < 2 && !rc; ++w) {
+                rc = encode_lbm(&map_src[w], fsrc, p->dtype, p->nx, p->ny, p->nz, bx + w * halo, by);
+                if (!rc) rc = encode_lbm(&map_dst[w], fdst, p->dtype, p->nx, p->ny, p->nz, bx + w * halo, by);
+            }
+            if (rc) return rc;
+            const size_t sb = lbm_pull_tma_stage_bytes(dt);
+            stages = p->opt_lbm_stages > 0 ? p->opt_lbm_stages : (dt == 0 ? 3 : 1);
+            if ((size_t)stages * sb > p->smem_optin) return fail(ST_EUNSUPPORTED, "LBM pull ring of %d stages", stages);
+            const int per_sm = std::max(1, std::min(2, (int)(p->smem_sm / ((size_t)stages * sb + 1024))));
+            const long long tiles = (long long)((p->nx + bx - 1) / bx) * ((p->ny + by - 1) / by) * p->nz;
+            tgrid = (int)std::min<long long>(tiles, (long long)p->sms * per_sm);
+            // tiles are dealt round-robin: a grid that is a multiple of the tile
+            // columns would give every CTA the same x position (and the CTAs holding
+            // the x walls all the slow bounce-back cells); one CTA fewer rotates them
+            const int tcols = (p->nx + bx - 1) / bx;
+            if (tgrid > 1 && tgrid % tcols == 0) --tgrid;
+        }
         // T + 1 passes; C in place when T is odd so the result lands in f_dst
         void* a = fsrc;
         void* b = fdst;
         auto pass = [&](int mode, void* from, void* to) -> int {
-            cudaError_t e = lbm_gather_launch(dt, p->exact, mode, from, to, p->fl2, prm, grid, p->stream);
+            cudaError_t e;
+            if (tma)
+                e = lbm_pull_tma_launch(dt, p->exact, mode, p->opt_pdl != 0, from == fsrc ? map_src : map_dst, from,
+                                        to, p->fl2, prm, tgrid, stages, p->stream);
+            else
+                e = lbm_gather_launch(dt, p->exact, mode, from, to, p->fl2, prm, grid, p->stream);
             if (e != cudaSuccess) return fail(ST_ECUDA, "lbm gather launch: %s", cudaGetErrorString(e));
             ++p->launches;
             return ST_OK;
@@ -1314,6 +1362,7 @@ static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T
         return ST_OK;
     }
     std::vector<int> ds = push ? std::vector<int>(T, 1) : sweep_depths(T, max_lbm_depth(p));
+    p->last_lbm_kernel = push ? 100 : 200 + max_lbm_depth(p);
     rc = run_sweeps(p, ds, fsrc, fdst, 19, flags, [&](const void* a, void* b, int d, const SlabView& sv) {
         if (push) return launch_lbm(p, a, b, sv.flags, omega, sv);
         return launch_lbm35(p, a, b, d, omega, sv);

@@ -255,3 +255,56 @@ def test_gather_form_kernels(oracle_lib, dtype, T):
             assert np.array_equal(got, ref)
         else:
             assert relerr(got, ref) <= TOL[dtype]
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+@pytest.mark.parametrize("shape", [(96, 50, 13), (64, 4, 5), (36, 9, 7), (128, 33, 10)])
+@pytest.mark.parametrize("T", [1, 2, 5])
+def test_gather_form_tma_pulls(oracle_lib, dtype, shape, T):
+    # ST_OPT_LBM_KERNEL 4: the gather form with the pull passes fed by TMA (shifted
+    # 4D boxes per population, shared-memory ring): bit-identical to the oracle in the
+    # exact build, within the gate otherwise; ragged tiles in x and y (36 x 9, 128 x 33),
+    # a single tile row (64 x 4), interior obstacle and LID cell, ring depths 1..6
+    nx, ny, nz = shape
+    flags = stgen.cavity_flags(nx, ny, nz)
+    flags[nz // 2, 2:4, 3:6] = stgen.WALL
+    flags[nz // 3, ny // 2, nx // 2] = stgen.LID
+    f0 = stgen.lbm_random(nx, ny, nz, 29, dtype)
+    ref = oracle_lib.lbm(f0, flags, 1.6, T)
+    for exact, stages in ((True, 0), (False, 0), (True, 1), (True, 3), (False, 5)):
+        with st.Plan(nx, ny, nz, torch.float32 if dtype == np.float32 else torch.float64, 1) as p:
+            p.set_bitexact(exact)
+            p.set_option(st.ST_OPT_LBM_KERNEL, 4)
+            if stages and (dtype == np.float32 or stages <= 4):
+                p.set_option(st.ST_OPT_LBM_STAGES, stages)
+            a = torch.from_numpy(f0).cuda()
+            b = torch.empty_like(a)
+            p.lbm(a, b, 1.6, T, torch.from_numpy(flags).cuda())
+            p.sync()
+            got = b.cpu().numpy()
+        if exact:
+            assert np.array_equal(got, ref), (exact, stages)
+        else:
+            assert relerr(got, ref) <= TOL[dtype]
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_gather_form_tma_pulls_256(oracle_lib, dtype):
+    # configs[2] size (256^3 cavity), random populations, T = 3, whole lattice
+    nx = ny = nz = 256
+    flags = stgen.cavity_flags(nx, ny, nz)
+    f0 = stgen.lbm_random(nx, ny, nz, 31, dtype)
+    ref = oracle_lib.lbm(f0, flags, 1.6, 3)
+    for exact in (True, False):
+        with st.Plan(nx, ny, nz, torch.float32 if dtype == np.float32 else torch.float64, 1) as p:
+            p.set_bitexact(exact)
+            p.set_option(st.ST_OPT_LBM_KERNEL, 4)
+            a = torch.from_numpy(f0).cuda()
+            b = torch.empty_like(a)
+            p.lbm(a, b, 1.6, 3, torch.from_numpy(flags).cuda())
+            p.sync()
+            got = b.cpu().numpy()
+        if exact:
+            assert np.array_equal(got, ref)
+        else:
+            assert relerr(got, ref) <= TOL[dtype]
