@@ -1321,13 +1321,13 @@ static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T
         int tgrid = 0, stages = 0;
         if (tma) {
             int bx, by, halo;
-            lbm_pull_tma_box(dt, &bx, &by, &halo);
+            lbm_pull_tma_box(dt, p->nx, &bx, &by, &halo);
             for (int w = 0; w < 2 && !rc; ++w) {
                 rc = encode_lbm(&map_src[w], fsrc, p->dtype, p->nx, p->ny, p->nz, bx + w * halo, by);
                 if (!rc) rc = encode_lbm(&map_dst[w], fdst, p->dtype, p->nx, p->ny, p->nz, bx + w * halo, by);
             }
             if (rc) return rc;
-            const size_t sb = lbm_pull_tma_stage_bytes(dt);
+            const size_t sb = lbm_pull_tma_stage_bytes(dt, p->nx);
             stages = p->opt_lbm_stages > 0 ? p->opt_lbm_stages : (dt == 0 ? 3 : 1);
             if ((size_t)stages * sb > p->smem_optin) return fail(ST_EUNSUPPORTED, "LBM pull ring of %d stages", stages);
             const int per_sm = std::max(1, std::min(2, (int)(p->smem_sm / ((size_t)stages * sb + 1024))));

@@ -51,8 +51,8 @@ cudaError_t lbm_gather_launch(int dtype, bool exact, int mode, const void* src, 
                               const LbmParams& p, int grid, cudaStream_t s);
 // TMA-fed pull pass of the gather form (lbm_tma.cu); maps = two 3D (x, y, 19 nz)
 // tensor maps of the source lattice, boxes (bx, by, 1) and (bx + halo, by, 1)
-size_t lbm_pull_tma_stage_bytes(int dtype);
-void lbm_pull_tma_box(int dtype, int* bx, int* by, int* halo);
+size_t lbm_pull_tma_stage_bytes(int dtype, int nx);
+void lbm_pull_tma_box(int dtype, int nx, int* bx, int* by, int* halo);
 // mode: LBM_COLLIDE / LBM_PULL / LBM_STREAM (the gather form's three passes)
 cudaError_t lbm_pull_tma_launch(int dtype, bool exact, int mode, bool pdl, const CUtensorMap* maps, const void* src,
                                 void* dst, const uint8_t* fl2, const LbmParams& p, int grid, int stages,

@@ -27,32 +27,27 @@
 // last pass skips the collision.
 #include "launch.h"
 
-#ifndef ST_LBM_TMA_CPT
-#define ST_LBM_TMA_CPT 1     // cells per consumer thread per tile (tile rows = 256 / BX * CPT)
-#endif
 #ifndef ST_LBM_TMA_PROBE
 #define ST_LBM_TMA_PROBE 0   // A/B probes only: 1 no collision, 2 no stores (results wrong)
 #endif
 
 namespace st35d {
 
-template <typename T> struct PullTile;
-template <typename T, int BX_, int BY_, int A_> struct PullGeom {
-    static constexpr int BX = BX_, BY = BY_, A = A_;
-    // a TMA destination must be 128-byte aligned: slots rounded up
+// tile of BX x BY = 256 cells (one per consumer thread), x halo A = 16 bytes;
+// a TMA destination must be 128-byte aligned, so population slots are rounded up
+template <typename T, int BX_> struct PullTile {
+    static constexpr int BX = BX_, BY = 256 / BX_, A = 16 / (int)sizeof(T);
     static constexpr int SLOT = ((BX + A) * BY * (int)sizeof(T) + 127) / 128 * 128 / (int)sizeof(T);
 };
-template <> struct PullTile<float> : PullGeom<float, 64, 4 * ST_LBM_TMA_CPT, 4> {};    // 256 B rows, 16 B halo
-template <> struct PullTile<double> : PullGeom<double, 32, 8 * ST_LBM_TMA_CPT, 2> {};
 
-constexpr int PULL_CONSUMERS = 256;   // consumer threads, ST_LBM_TMA_CPT cells each per tile
+constexpr int PULL_CONSUMERS = 256;   // consumer threads, one cell each per tile
 constexpr int PULL_THREADS = PULL_CONSUMERS + 32;
 
 // population i's box: width BX (ex = 0) or BX + A (ex = +-1: the 16-byte x halo
 // on the upstream side), row pitch = box width; cell column cx reads column
 // col0 + cx of the box
-template <typename T, int I> struct PullBox {
-    static constexpr int BX = PullTile<T>::BX, A = PullTile<T>::A;
+template <typename G, int I> struct PullBox {
+    static constexpr int BX = G::BX, A = G::A;
     static constexpr int ex = D3Q19<I>::ex;
     static constexpr int pitch = ex == 0 ? BX : BX + A;
     static constexpr int xoff = ex > 0 ? -A : 0;          // box start relative to x0
@@ -62,15 +57,16 @@ template <typename T, int I> struct PullBox {
 // MODE (lbm_kernel.cuh): LBM_PULL = stream + collide (the hot pass), LBM_COLLIDE =
 // collide only (unshifted boxes; may run in place, src == dst), LBM_STREAM =
 // stream only.  The first and last pass of the gather form run the same kernel.
-template <typename T, bool E, int MODE>
+template <typename T, bool E, int MODE, int TBX>
 __global__ void __launch_bounds__(PULL_THREADS, 2)
 lbm_pull_tma_kernel(const __grid_constant__ CUtensorMap mapn, const __grid_constant__ CUtensorMap mapw,
                     const T* src, T* dst, const uint8_t* __restrict__ fl2, const LbmParams p,
                     int stages, int tiles_x, int tiles_y) {
-    constexpr int BX = PullTile<T>::BX, BY = PullTile<T>::BY, A = PullTile<T>::A, NC = PULL_CONSUMERS;
-    constexpr int CPT = ST_LBM_TMA_CPT, RB = NC / BX;   // sub-rows of RB rows, one per pass
+    using G = PullTile<T, TBX>;
+    constexpr int BX = G::BX, BY = G::BY, A = G::A, NC = PULL_CONSUMERS;
+    constexpr int CPT = 1, RB = NC / BX;          // (one cell per consumer thread)
     static_assert(RB * CPT == BY, "tile rows");
-    constexpr int SLOT = PullTile<T>::SLOT;       // elements reserved per population box (128-byte aligned)
+    constexpr int SLOT = G::SLOT;                 // elements reserved per population box (128-byte aligned)
     constexpr uint32_t NB = BX * BY * sizeof(T), WB = (BX + A) * BY * sizeof(T);
     constexpr uint32_t TX_INTERIOR = 9 * NB + 10 * WB, TX_SHELL = 19 * NB;   // 9 populations with ex = 0
     extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -122,7 +118,7 @@ lbm_pull_tma_kernel(const __grid_constant__ CUtensorMap mapn, const __grid_const
                     mbar_arrive_expect_tx(&full[s], TX_INTERIOR);
                     [&]<int... Is>(std::integer_sequence<int, Is...>) {
                         ((tma_load_3d(b + Is * SLOT, D3Q19<Is>::ex == 0 ? &mapn : &mapw, &full[s],
-                                      x0 + PullBox<T, Is>::xoff, y0 - D3Q19<Is>::ey, Is * nz + z - D3Q19<Is>::ez)),
+                                      x0 + PullBox<G, Is>::xoff, y0 - D3Q19<Is>::ey, Is * nz + z - D3Q19<Is>::ez)),
                          ...);
                     }(std::make_integer_sequence<int, 19>{});
                 }
@@ -172,7 +168,7 @@ lbm_pull_tma_kernel(const __grid_constant__ CUtensorMap mapn, const __grid_const
             for (int i = 0; i < 19; ++i) f[i] = b[i * SLOT + cy * BX + cx];
         } else {
             [&]<int... Is>(std::integer_sequence<int, Is...>) {
-                ((f[Is] = b[Is * SLOT + cy * PullBox<T, Is>::pitch + PullBox<T, Is>::col0 + cx]), ...);
+                ((f[Is] = b[Is * SLOT + cy * PullBox<G, Is>::pitch + PullBox<G, Is>::col0 + cx]), ...);
             }(std::make_integer_sequence<int, 19>{});
         }
         // every consumer thread releases the stage itself (after its last sub-row),
@@ -230,41 +226,50 @@ lbm_pull_tma_kernel(const __grid_constant__ CUtensorMap mapn, const __grid_const
     }
 }
 
-template <typename T>
-size_t lbm_pull_stage_bytes() { return 19u * PullTile<T>::SLOT * sizeof(T); }
+// tile width for a lattice row of nx cells (measured on B200, FP32 cavity, GLUPS:
+// 256^3 64 x 4 34.1 vs 128 x 2 30.8; 1024^3 64 x 4 25.0 vs 128 x 2 30.0)
+static int pull_bx(int dtype, int nx) { return dtype == 0 ? (nx >= 512 ? 128 : 64) : 32; }
 
-template <typename T, bool E>
+template <typename T, int BX>
+static size_t stage_bytes() { return 19u * PullTile<T, BX>::SLOT * sizeof(T); }
+
+template <typename T, bool E, int BX>
 static cudaError_t pull_t(int mode, bool pdl, const CUtensorMap* maps, const void* src, void* dst,
                           const uint8_t* fl2, const LbmParams& p, int grid, int stages, cudaStream_t s) {
-    auto k = mode == LBM_COLLIDE ? lbm_pull_tma_kernel<T, E, LBM_COLLIDE>
-           : mode == LBM_STREAM  ? lbm_pull_tma_kernel<T, E, LBM_STREAM> : lbm_pull_tma_kernel<T, E, LBM_PULL>;
-    const size_t smem = (size_t)stages * (lbm_pull_stage_bytes<T>() + 16);
+    auto k = mode == LBM_COLLIDE ? lbm_pull_tma_kernel<T, E, LBM_COLLIDE, BX>
+           : mode == LBM_STREAM  ? lbm_pull_tma_kernel<T, E, LBM_STREAM, BX> : lbm_pull_tma_kernel<T, E, LBM_PULL, BX>;
+    const size_t smem = (size_t)stages * (stage_bytes<T, BX>() + 16);
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    const int tiles_x = (p.nx + PullTile<T>::BX - 1) / PullTile<T>::BX;
-    const int tiles_y = (p.ny + PullTile<T>::BY - 1) / PullTile<T>::BY;
+    const int tiles_x = (p.nx + PullTile<T, BX>::BX - 1) / PullTile<T, BX>::BX;
+    const int tiles_y = (p.ny + PullTile<T, BX>::BY - 1) / PullTile<T, BX>::BY;
     return launch_pdl(pdl, k, grid, PULL_THREADS, smem, s, maps[0], maps[1], static_cast<const T*>(src),
                       static_cast<T*>(dst), fl2, p, stages, tiles_x, tiles_y);
 }
 
-size_t lbm_pull_tma_stage_bytes(int dtype) {
-    return (dtype == 0 ? lbm_pull_stage_bytes<float>() : lbm_pull_stage_bytes<double>()) + 16;
+size_t lbm_pull_tma_stage_bytes(int dtype, int nx) {
+    const int bx = pull_bx(dtype, nx);
+    return (dtype == 1 ? stage_bytes<double, 32>() : bx == 128 ? stage_bytes<float, 128>() : stage_bytes<float, 64>())
+           + 16;
 }
 
-void lbm_pull_tma_box(int dtype, int* bx, int* by, int* halo) {
-    *bx = dtype == 0 ? PullTile<float>::BX : PullTile<double>::BX;
-    *by = dtype == 0 ? PullTile<float>::BY : PullTile<double>::BY;
-    *halo = dtype == 0 ? PullTile<float>::A : PullTile<double>::A;
+void lbm_pull_tma_box(int dtype, int nx, int* bx, int* by, int* halo) {
+    *bx = pull_bx(dtype, nx);
+    *by = 256 / *bx;
+    *halo = dtype == 0 ? 4 : 2;
 }
 
 // maps[0]: box (BX, BY, 1), maps[1]: box (BX + A, BY, 1) over the source lattice as (x, y, 19 nz)
 cudaError_t lbm_pull_tma_launch(int dtype, bool exact, int mode, bool pdl, const CUtensorMap* maps, const void* src,
                                 void* dst, const uint8_t* fl2, const LbmParams& p, int grid, int stages,
                                 cudaStream_t s) {
-    if (dtype == 0) return exact ? pull_t<float, true>(mode, pdl, maps, src, dst, fl2, p, grid, stages, s)
-                                 : pull_t<float, false>(mode, pdl, maps, src, dst, fl2, p, grid, stages, s);
-    return exact ? pull_t<double, true>(mode, pdl, maps, src, dst, fl2, p, grid, stages, s)
-                 : pull_t<double, false>(mode, pdl, maps, src, dst, fl2, p, grid, stages, s);
+    if (dtype == 1) return exact ? pull_t<double, true, 32>(mode, pdl, maps, src, dst, fl2, p, grid, stages, s)
+                                 : pull_t<double, false, 32>(mode, pdl, maps, src, dst, fl2, p, grid, stages, s);
+    if (pull_bx(dtype, p.nx) == 128)
+        return exact ? pull_t<float, true, 128>(mode, pdl, maps, src, dst, fl2, p, grid, stages, s)
+                     : pull_t<float, false, 128>(mode, pdl, maps, src, dst, fl2, p, grid, stages, s);
+    return exact ? pull_t<float, true, 64>(mode, pdl, maps, src, dst, fl2, p, grid, stages, s)
+                 : pull_t<float, false, 64>(mode, pdl, maps, src, dst, fl2, p, grid, stages, s);
 }
 
 }  // namespace st35d

@@ -258,13 +258,14 @@ def test_gather_form_kernels(oracle_lib, dtype, T):
 
 
 @pytest.mark.parametrize("dtype", [np.float32, np.float64])
-@pytest.mark.parametrize("shape", [(96, 50, 13), (64, 4, 5), (36, 9, 7), (128, 33, 10)])
+@pytest.mark.parametrize("shape", [(96, 50, 13), (64, 4, 5), (36, 9, 7), (128, 33, 10), (520, 5, 6)])
 @pytest.mark.parametrize("T", [1, 2, 5])
 def test_gather_form_tma_pulls(oracle_lib, dtype, shape, T):
     # ST_OPT_LBM_KERNEL 4: the gather form with the pull passes fed by TMA (shifted
     # 4D boxes per population, shared-memory ring): bit-identical to the oracle in the
     # exact build, within the gate otherwise; ragged tiles in x and y (36 x 9, 128 x 33),
-    # a single tile row (64 x 4), interior obstacle and LID cell, ring depths 1..6
+    # a single tile row (64 x 4), the 128-wide FP32 tiles of rows >= 512 cells (520 x 5),
+    # interior obstacle and LID cell, ring depths 1..5
     nx, ny, nz = shape
     flags = stgen.cavity_flags(nx, ny, nz)
     flags[nz // 2, 2:4, 3:6] = stgen.WALL
