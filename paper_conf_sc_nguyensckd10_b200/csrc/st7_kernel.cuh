@@ -445,6 +445,12 @@ st7_35d_kernel(const __grid_constant__ CUtensorMap tmap, const St7Params p) {
     while (item < item_end) {
         const Seg sg = seg_at(item);
 #ifdef ST7_TRACE
+        if (nseg_tr == 0) {
+            unsigned smid;
+            asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+            ST7_STAMP(15, (unsigned long long)sg.tile | ((unsigned long long)smid << 16) |
+                              ((unsigned long long)sg.za << 32));
+        }
         if (nseg_tr < 3) ST7_STAMP(2 + 3 * nseg_tr, st7_gtime());
         if (nseg_tr < 3) ST7_STAMP(14, (nseg_tr ? st7_trace_buf[blockIdx.x][14] : 0ull) |
                                            ((unsigned long long)(sg.zb - sg.za) << (16 * nseg_tr)));

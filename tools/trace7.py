@@ -41,6 +41,27 @@ for c in sys.argv[1:]:
             pro.append(s1 - s0); stdy.append((s2 - s1) / max(Lj, 1)); epi.append(e - s2); Ls.append(Lj)
     pro, stdy, epi, Ls = (np.array(v, float) for v in (pro, stdy, epi, Ls))
     info = p.info()
+    Ltot = np.array([sum((int(b[i, 14]) >> (16 * j)) & 0xffff for j in range(min(int(ns[i]), 3))) for i in range(G)])
+    order = np.argsort(-busy)
+    print("   slowest CTAs (busy us, segments, planes, go us):",
+          [(round(busy[i] / 1e3, 1), int(ns[i]), int(Ltot[i]), round(go[i] / 1e3, 2)) for i in order[:8]])
+    tile0 = b[:, 15] & 0xffff
+    smid = (b[:, 15] >> 16) & 0xffff
+    print("   slowest (tile, smid):", [(int(tile0[i]), int(smid[i])) for i in order[:12]])
+    print("   fastest (tile, smid):", [(int(tile0[i]), int(smid[i])) for i in order[-12:]])
+    tb = {}
+    for i in range(G):
+        if ns[i] == 1:
+            tb.setdefault(int(tile0[i]), []).append(busy[i] / 1e3)
+    print("   1-seg busy by tile:", {t: round(float(np.median(v)), 1) for t, v in sorted(tb.items())})
+    half = smid < 74
+    print(f"   busy med smid<74 {np.median(busy[half & (ns == 1)])/1e3:.1f}  smid>=74 {np.median(busy[~half & (ns == 1)])/1e3:.1f}")
+    print("   fastest CTAs:", [(round(busy[i] / 1e3, 1), int(ns[i]), int(Ltot[i])) for i in order[-6:]])
+    for k in (1, 2):
+        m = ns == k
+        if m.any():
+            print(f"   {k}-segment CTAs: {m.sum()}  busy med {np.median(busy[m])/1e3:.1f} us  planes med {np.median(Ltot[m]):.0f}"
+                  f"  us/plane-equiv {np.median(busy[m] / Ltot[m])/1e3:.3f}")
     print(f"   tiles {info['tiles_x']}x{info['tiles_y']} thr {info['threads']}  segments timed {len(Ls)}  L med {np.median(Ls):.0f}"
           f"  prolog us med {np.median(pro)/1e3:.2f} (max {pro.max()/1e3:.2f})  steady us/plane med {np.median(stdy)/1e3:.3f}"
           f"  epilog us med {np.median(epi)/1e3:.2f}")
