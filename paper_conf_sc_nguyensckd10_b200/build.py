@@ -51,6 +51,7 @@ UNITS = [
     ("naive.cu", "naive.o", []),
     ("st27.cu", "st27.o", []),
     ("st13_inst.cu", "st13_inst.o", []),
+    ("st27t_inst.cu", "st27t_inst.o", []),
     ("model.cpp", "model.o", []),
 ] + [
     ("st7_inst.cu", f"st7_{tn}_{mode}.o", [f"-DST_T={t}", f"-DST_TNAME={tn}", f"-DST_EXACT={ex}"])

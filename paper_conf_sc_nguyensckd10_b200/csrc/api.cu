@@ -14,6 +14,7 @@
 #include "launch.h"
 #include "dist.h"
 #include "st13_kernel.cuh"
+#include "st27t_kernel.cuh"
 
 using namespace st35d;
 
@@ -99,6 +100,7 @@ struct Geo7 {
     double kappa = 0;
     St7LaunchFn fn = nullptr;
     St13LaunchFn fn13 = nullptr;             // radius-2 plans
+    St27tLaunchFn fn27t = nullptr;           // 27-point plans (tolerance build)
 };
 
 struct st_plan {
@@ -317,6 +319,53 @@ static int plan13(st_plan* p, int d, int nzo, Geo7& g) {
     g.kappa = (double)g.tiles_x * g.TX * g.tiles_y * g.TY / ((double)p->nx * p->ny);
     g.fn13 = st13_lookup(p->dtype == ST_F32 ? 0 : 1, p->exact, d, g.VY);
     if (!g.fn13) return fail(ST_EUNSUPPORTED, "no radius-2 kernel for dim_T %d", d);
+    return ST_OK;
+}
+
+// ----------------------------------------------------------------------------
+// 27-point planner (st27t_kernel.cuh, tolerance build): the 7-point planner with
+// R = 1 and the exchange double-buffered by round parity; VY = 4 rows per thread
+// up to depth vy4_max, else 2
+// ----------------------------------------------------------------------------
+static size_t smem27t(const Geo7& g, st_dtype dt, int ring) {
+    return (size_t)ring * g.TX * g.TY * esize(dt) + (size_t)(g.d > 1 ? g.d - 1 : 0) * 4 * g.threads * 16 +
+           ST7_RING_MAX * 8;
+}
+
+static int plan27t(st_plan* p, int d, int nzo, Geo7& g) {
+    g.d = d;
+    g.VX = p->dtype == ST_F32 ? 4 : 2;
+    g.NTX = p->dtype == ST_F32 ? 16 : 32;
+    g.TX = g.NTX * g.VX;
+    g.VY = d <= ST27T_VY4_MAX ? 4 : 2;
+    g.maxt = 256;
+    g.minb = 1;
+    g.hx = (d + g.VX - 1) / g.VX * g.VX;
+    g.wx = (g.TX - g.hx - d) & ~(g.VX - 1);
+    if (g.wx < g.VX) return fail(ST_EUNSUPPORTED, "27-point: dim_T %d too deep for the %d-wide tile", d, g.TX);
+    g.tiles_x = (p->nx + g.wx - 1) / g.wx;
+    long best = -1;
+    for (int nty = 2; nty <= g.maxt / g.NTX; ++nty) {
+        Geo7 c = g;
+        c.NTY = nty;
+        c.TY = nty * c.VY;
+        c.threads = c.NTX * nty;
+        if (c.TY - 2 * d < 1) continue;
+        place_y(c, p->ny, d, 1);
+        c.ring = 0;
+        for (int r = ST7_RING_MAX; r >= 4; --r)
+            if (smem27t(c, p->dtype, r) <= p->smem_optin) { c.ring = r; break; }
+        if (c.ring < 4) continue;
+        c.smem = smem27t(c, p->dtype, c.ring);
+        const long cost = (long)c.tiles_y * c.TY;
+        if (best < 0 || cost < best || (cost == best && c.TY > g.TY)) { best = cost; g = c; }
+    }
+    if (best < 0) return fail(ST_EUNSUPPORTED, "27-point: dim_T %d too deep for the tiles of this build", d);
+    const long long work = (long long)g.tiles_x * g.tiles_y * nzo;
+    g.grid = (int)std::min<long long>(p->sms, std::max<long long>(work, 1));
+    g.kappa = (double)g.tiles_x * g.TX * g.tiles_y * g.TY / ((double)p->nx * p->ny);
+    g.fn27t = st27t_lookup(p->dtype == ST_F32 ? 0 : 1, d, g.VY);
+    if (!g.fn27t) return fail(ST_EUNSUPPORTED, "no 27-point kernel for dim_T %d", d);
     return ST_OK;
 }
 
@@ -898,6 +947,33 @@ extern "C" int st7_run(st_plan* p, const void* in, void* out, double alpha, doub
 // 27-point stencil: ceil(T/D) ping-pong sweeps of the
 // st27.cu kernel, D = min(dim_T, st27_depth_max()); single process only.
 // ----------------------------------------------------------------------------
+static int launch27t(st_plan* p, const void* src, void* dst, int d, const double w[4]) {
+    Geo7 g;
+    int rc = plan27t(p, d, p->nz, g);
+    if (rc) return rc;
+    CUtensorMap map;
+    rc = encode_3d(&map, src, p->dtype, p->nx, p->ny, p->nz, g.TX, g.TY);
+    if (rc) return rc;
+    St27tParams prm{};
+    St7Params& q = prm.g;
+    q.out = dst;
+    q.nx = p->nx; q.ny = p->ny; q.nzb = p->nz; q.zbase = 0; q.nzg = p->nz;
+    q.za = 0; q.zb = p->nz;
+    q.tiles_x = g.tiles_x; q.ntiles = g.tiles_x * g.tiles_y;
+    q.wx = g.wx; q.wy = g.wy; q.hx = g.hx;
+    q.tiles_y = g.tiles_y; q.ey = g.ey; q.ly_last = g.ly_last; q.oy0_last = g.oy0_last;
+    q.ring = g.ring;
+    q.pdl = p->opt_pdl;
+    q.alpha = w[0]; q.beta = w[1]; prm.gamma = w[2]; prm.delta = w[3];
+    if ((long long)q.ntiles * p->nz >= (1LL << 31)) return fail(ST_EUNSUPPORTED, "grid too large");
+    const int grid = std::min(g.grid, ST7_MAX_GRID);
+    split_work(q.ntiles, p->nz, d, grid, q.split);   // restart: 2d-1 prolog rounds
+    cudaError_t e = g.fn27t(&map, prm, grid, g.threads, g.smem, p->stream);
+    if (e != cudaSuccess) return fail(ST_ECUDA, "st27t launch (d=%d): %s", d, cudaGetErrorString(e));
+    ++p->launches;
+    return ST_OK;
+}
+
 static int run27_device(st_plan* p, const void* in, void* out, const double w[4], int T) {
     const size_t n = (size_t)p->nx * p->ny * p->nz * esize(p->dtype);
     p->launches = 0;
@@ -905,10 +981,17 @@ static int run27_device(st_plan* p, const void* in, void* out, const double w[4]
         CUDA_TRY(cudaMemcpyAsync(out, in, n, cudaMemcpyDeviceToDevice, p->stream));
         return ST_OK;
     }
-    const int D = std::min(p->dimT, st27_depth_max(p->dtype == ST_F32 ? 0 : 1));
+    // tolerance build: the 7-point machinery (st27t); bit-exact build: the oracle-order kernel (st27.cu)
+    const bool tk = !p->exact;
+    const int D = std::min(p->dimT, tk ? ST27T_MAX_DIM_T : st27_depth_max(p->dtype == ST_F32 ? 0 : 1));
     const std::vector<int> ds = sweep_depths(T, D);
     void* bufs[2] = {const_cast<void*>(in), out};
     for (size_t k = 0; k < ds.size(); ++k) {
+        if (tk) {
+            int rc = launch27t(p, bufs[k % 2], bufs[(k + 1) % 2], ds[k], w);
+            if (rc) return rc;
+            continue;
+        }
         cudaError_t e = st27_launch(p->dtype == ST_F32 ? 0 : 1, p->exact, ds[k], bufs[k % 2], bufs[(k + 1) % 2], p->nx,
                                     p->ny, p->nz, w[0], w[1], w[2], w[3], p->sms, p->stream, nullptr);
         if (e != cudaSuccess) return fail(ST_ECUDA, "st27 launch: %s", cudaGetErrorString(e));

@@ -44,6 +44,19 @@ using St13LaunchFn = cudaError_t (*)(const CUtensorMap* map, const St13Params& p
 St13LaunchFn st13_lookup(int dtype, bool exact, int D, int VY);
 constexpr int ST13_MAX_DIM_T = 4;
 
+// 27-point sweep on the 7-point machinery (st27t_kernel.cuh, tolerance build);
+// nullptr if (D, VY) is not compiled
+struct St27tParams;
+using St27tLaunchFn = cudaError_t (*)(const CUtensorMap* map, const St27tParams& p, int grid, int threads,
+                                      size_t smem, cudaStream_t s);
+St27tLaunchFn st27t_lookup(int dtype, int D, int VY);
+constexpr int ST27T_MAX_DIM_T = 4;
+#ifndef ST27T_VY4_MAX_AB
+constexpr int ST27T_VY4_MAX = 1;   // VY = 4 rows per thread up to this depth, else 2
+#else
+constexpr int ST27T_VY4_MAX = ST27T_VY4_MAX_AB;   // A/B tuning builds only
+#endif
+
 bool lbm_push_batched(int esize, int nx, int ny, int nzb, int force);   // kernel choice (also sets the grid)
 cudaError_t lbm_push_launch(int dtype, bool exact, bool slab, bool batched, const void* src, void* dst,
                             const uint8_t* fl2, const LbmParams& p, int grid, cudaStream_t s);

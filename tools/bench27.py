@@ -8,7 +8,7 @@ import paper_conf_sc_nguyensckd10_b200 as st
 
 n = int(sys.argv[1]) if len(sys.argv) > 1 else 256
 T = 100
-for dt_np, tdt, dmax in ((np.float32, torch.float32, 4), (np.float64, torch.float64, 2)):
+for dt_np, tdt, dmax in ((np.float32, torch.float32, 4), (np.float64, torch.float64, 4)):
     x = torch.from_numpy(stgen.grid7(n, n, n, 2, dt_np)).cuda()
     y = torch.empty_like(x)
     for d in range(1, dmax + 1):
