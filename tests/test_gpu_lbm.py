@@ -155,6 +155,7 @@ def test_config4_lbm_1024_light_cone(oracle_lib):
     # small cavity with the same local geometry; every shifted window has its light cone
     # inside both lattices.  Fluid mass is conserved (P8b) over the whole lattice.
     n, T = 1024, 3
+    torch.cuda.empty_cache()
     need = 2 * 19 * n ** 3 * 4 + 3 * n ** 3 + (4 << 30)
     if torch.cuda.mem_get_info()[0] < need:
         pytest.skip("1024^3 FP32 lattice pair does not fit this device")
@@ -189,6 +190,74 @@ def test_config4_lbm_1024_light_cone(oracle_lib):
         for z0 in range(1, n - 1, 64):
             mass += float(g[i, z0:min(z0 + 64, n - 1), 1:n - 1, 1:n - 1].double().sum())
     assert abs(mass - mass0) <= 1e-6 * mass0
+
+
+def test_config4_lbm_1024_random_windows(oracle_lib):
+    # configs[4] lattice (1024^3 FP32 cavity) with RANDOM populations through the
+    # automatic kernel choice (the TMA gather form with 128 x 2 tiles), bit-exact and
+    # tolerance builds.  After T steps a cell depends only on its radius-T
+    # neighbourhood, so windows are checked against the oracle run on a crop of the
+    # same input: the crop keeps the real lattice faces and closes its cut faces
+    # with WALL cells, and only cells farther than T + 1 from a cut face are
+    # compared.  Windows: centre, lid centre, a bottom corner, the x = 0 wall, and a
+    # seam of the 128-wide x tiles / 2-row y tiles.
+    n, T, k = 1024, 5, 3   # T >= 4: the automatic choice is the gather form (T + 1 passes, odd: in-place collide)
+    import gc
+    gc.collect()
+    torch.cuda.empty_cache()   # the previous 1024^3 test's lattices stay cached otherwise
+    need = 2 * 19 * n ** 3 * 4 + 3 * n ** 3 + (4 << 30)
+    if torch.cuda.mem_get_info()[0] < need:
+        pytest.skip("1024^3 FP32 lattice pair does not fit this device")
+    f, fl = _cavity_on_device(n, torch.float32)   # f is refilled with random populations below
+    g = torch.empty_like(f)
+    w = stgen.lbm_rest(1, 1, 1, np.float32).reshape(19)
+    centres = [(512, 512, 512), (512, n - 1, 512), (0, 0, 0), (300, 700, 0), (77, 301, 128)]   # (z, y, x)
+    m = k + T + 1
+    crops = []
+    for c in centres:
+        lo = [max(0, v - m) for v in c]
+        hi = [min(n, v + m + 1) for v in c]
+        crops.append((lo, hi))
+
+    def fill():
+        gen = torch.Generator(device="cuda")
+        gen.manual_seed(1234)
+        for i in range(19):
+            f[i].uniform_(-1.0, 1.0, generator=gen).mul_(0.1).add_(1.0).mul_(float(w[i]))
+        torch.cuda.synchronize()
+
+    for exact in (True, False):
+        fill()
+        inputs = [f[:, lo[0]:hi[0], lo[1]:hi[1], lo[2]:hi[2]].cpu().numpy() for lo, hi in crops]
+        with st.Plan(n, n, n, torch.float32, 1) as p:
+            p.set_lid(0.05, 0.0, 0.0)
+            p.set_bitexact(exact)
+            p.lbm(f, g, 1.6, T, fl)
+            p.sync()
+            assert p.info(True)["kernel"] == 400
+        for (lo, hi), c, f0 in zip(crops, centres, inputs):
+            flc = fl[lo[0]:hi[0], lo[1]:hi[1], lo[2]:hi[2]].cpu().numpy().copy()
+            # cut faces (inside the lattice) become WALL
+            if lo[0] > 0: flc[0] = stgen.WALL
+            if hi[0] < n: flc[-1] = stgen.WALL
+            if lo[1] > 0: flc[:, 0] = stgen.WALL
+            if hi[1] < n: flc[:, -1] = stgen.WALL
+            if lo[2] > 0: flc[:, :, 0] = stgen.WALL
+            if hi[2] < n: flc[:, :, -1] = stgen.WALL
+            ref = oracle_lib.lbm(f0, flc, 1.6, T)
+            # compared: cells farther than T + 1 from every cut face
+            sl = []
+            for d in range(3):
+                a = (T + 2) if lo[d] > 0 else 0
+                b = (hi[d] - lo[d]) - ((T + 2) if hi[d] < n else 0)
+                sl.append(slice(a, b))
+            got = g[:, lo[0]:hi[0], lo[1]:hi[1], lo[2]:hi[2]].cpu().numpy()
+            gw, rw = got[(slice(None),) + tuple(sl)], ref[(slice(None),) + tuple(sl)]
+            assert gw.size > 0
+            if exact:
+                assert np.array_equal(gw, rw), c
+            else:
+                assert relerr(gw, rw) <= TOL[np.float32], c
 
 
 @pytest.mark.parametrize("shape", [(4, 3, 3), (4, 3, 5), (8, 7, 3), (40, 3, 9)])
