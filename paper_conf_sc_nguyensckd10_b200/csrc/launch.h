@@ -51,11 +51,9 @@ using St27tLaunchFn = cudaError_t (*)(const CUtensorMap* map, const St27tParams&
                                       size_t smem, cudaStream_t s);
 St27tLaunchFn st27t_lookup(int dtype, int D, int VY);
 constexpr int ST27T_MAX_DIM_T = 4;
-#ifndef ST27T_VY4_MAX_AB
-constexpr int ST27T_VY4_MAX = 1;   // VY = 4 rows per thread up to this depth, else 2
-#else
-constexpr int ST27T_VY4_MAX = ST27T_VY4_MAX_AB;   // A/B tuning builds only
-#endif
+// VY = 4 rows per thread up to this depth, else 2 (measured 256^3 FP32 dim_T 2: VY 2 623,
+// VY 4 524 Gupd/s -- 255 registers with spills)
+constexpr int ST27T_VY4_MAX = 1;
 
 bool lbm_push_batched(int esize, int nx, int ny, int nzb, int force);   // kernel choice (also sets the grid)
 cudaError_t lbm_push_launch(int dtype, bool exact, bool slab, bool batched, const void* src, void* dst,

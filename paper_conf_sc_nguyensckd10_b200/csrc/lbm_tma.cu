@@ -27,9 +27,6 @@
 // last pass skips the collision.
 #include "launch.h"
 
-#ifndef ST_LBM_TMA_PROBE
-#define ST_LBM_TMA_PROBE 0   // A/B probes only: 1 no collision, 2 no stores (results wrong)
-#endif
 
 namespace st35d {
 
@@ -64,8 +61,7 @@ lbm_pull_tma_kernel(const __grid_constant__ CUtensorMap mapn, const __grid_const
                     int stages, int tiles_x, int tiles_y) {
     using G = PullTile<T, TBX>;
     constexpr int BX = G::BX, BY = G::BY, A = G::A, NC = PULL_CONSUMERS;
-    constexpr int CPT = 1, RB = NC / BX;          // (one cell per consumer thread)
-    static_assert(RB * CPT == BY, "tile rows");
+    static_assert(NC == BX * BY, "one consumer thread per tile cell");
     constexpr int SLOT = G::SLOT;                 // elements reserved per population box (128-byte aligned)
     constexpr uint32_t NB = BX * BY * sizeof(T), WB = (BX + A) * BY * sizeof(T);
     constexpr uint32_t TX_INTERIOR = 9 * NB + 10 * WB, TX_SHELL = 19 * NB;   // 9 populations with ex = 0
@@ -130,38 +126,28 @@ lbm_pull_tma_kernel(const __grid_constant__ CUtensorMap mapn, const __grid_const
     const size_t plane = (size_t)nx * ny;
     const size_t nc = plane * nz;
     const T omega = T(p.omega);
-    const int cx = tid % BX, cy0 = tid / BX;
-    // the cells' flags are read one tile ahead (their latency off the tile's critical path)
-    uint32_t fl_next[CPT];
-    auto flags_of = [&](long long tile) {
+    const int cx = tid % BX, cy = tid / BX;
+    // the cell's flag is read one tile ahead (its latency off the tile's critical path)
+    auto flag_of = [&](long long tile) -> uint32_t {
         int x0, y0, z;
         where(tile, x0, y0, z);
-#pragma unroll
-        for (int j = 0; j < CPT; ++j) {
-            const int x = x0 + cx, y = y0 + cy0 + j * RB;
-            fl_next[j] = x < nx && y < ny ? (uint32_t)fl2[(size_t)z * plane + (size_t)y * nx + x] : 0u;
-        }
+        const int x = x0 + cx, y = y0 + cy;
+        return x < nx && y < ny ? (uint32_t)fl2[(size_t)z * plane + (size_t)y * nx + x] : 0u;
     };
-    if (t_begin < t_end) flags_of(t_begin);
+    uint32_t fl_next = t_begin < t_end ? flag_of(t_begin) : 0u;
     int k = 0;
     for (long long tile = t_begin; tile < t_end; tile += t_step, ++k) {
         const int s = k % stages;
         int x0, y0, z;
         where(tile, x0, y0, z);
-        uint32_t fls[CPT];
-#pragma unroll
-        for (int j = 0; j < CPT; ++j) fls[j] = fl_next[j];
-        if (tile + t_step < t_end) flags_of(tile + t_step);
-        const bool own = MODE == LBM_COLLIDE || z == 0 || z == nz - 1;
-        mbar_wait(&full[s], (k / stages) & 1);
-        const T* b = buf + (size_t)s * 19 * SLOT;
-#pragma unroll 1
-        for (int j = 0; j < CPT; ++j) {
-        const int cy = cy0 + j * RB;
+        const uint32_t fl = fl_next;
+        if (tile + t_step < t_end) fl_next = flag_of(tile + t_step);
+        const bool own = MODE == LBM_COLLIDE || z == 0 || z == nz - 1;   // unshifted boxes
         const int x = x0 + cx, y = y0 + cy;
         const bool inb = x < nx && y < ny;
         const size_t c = (size_t)z * plane + (size_t)y * nx + x;
-        const uint32_t fl = fls[j];
+        mbar_wait(&full[s], (k / stages) & 1);
+        const T* b = buf + (size_t)s * 19 * SLOT;
         T f[19];
         if (own) {
 #pragma unroll
@@ -171,16 +157,14 @@ lbm_pull_tma_kernel(const __grid_constant__ CUtensorMap mapn, const __grid_const
                 ((f[Is] = b[Is * SLOT + cy * PullBox<G, Is>::pitch + PullBox<G, Is>::col0 + cx]), ...);
             }(std::make_integer_sequence<int, 19>{});
         }
-        // every consumer thread releases the stage itself (after its last sub-row),
-        // behind a generic->async proxy fence: the stage is next written by TMA
-        // (async proxy), and the thread's shared-memory reads (generic proxy) must
-        // be complete first.  Measured on B200 without the fence (release-semantics
-        // arrive alone, or one arrive per warp after __syncwarp): the next TMA write
-        // overtook reads still in flight — wrong cells on 256^3 FP64, 2 CTAs per SM.
-        if (j == CPT - 1) {
-            fence_proxy_async();
-            mbar_arrive(&empty[s]);
-        }
+        // every consumer thread releases the stage itself, behind a generic->async
+        // proxy fence: the stage is next written by TMA (async proxy), and the
+        // thread's shared-memory reads (generic proxy) must be complete first.
+        // Measured on B200 without the fence (release-semantics arrive alone, or one
+        // arrive per warp after __syncwarp): the next TMA write overtook reads still
+        // in flight — wrong cells on 256^3 FP64 with 2 CTAs per SM.
+        fence_proxy_async();
+        mbar_arrive(&empty[s]);
         if (!inb) continue;
         if (fl & 0x7fu) {   // WALL / LID: copied through (own values; unshifted tiles already hold them)
             if (!own) {
@@ -192,37 +176,31 @@ lbm_pull_tma_kernel(const __grid_constant__ CUtensorMap mapn, const __grid_const
                 // the 18 upstream flags and the cell's own 18 values are loaded together
                 // (one memory round trip), then selected
                 uint32_t sf[19];
-                T own[19];
+                T mine[19];
                 [&]<int... Is>(std::integer_sequence<int, Is...>) {
                     ((sf[Is] = Is == 0 ? 0u
                                        : (uint32_t)__ldg(fl2 + (long long)c -
                                                          ((long long)D3Q19<Is>::ex + (long long)D3Q19<Is>::ey * nx +
                                                           (long long)D3Q19<Is>::ez * (long long)plane))),
                      ...);
-                    ((own[Is] = Is == 0 ? T(0) : src[(size_t)D3Q19<Is>::opp * nc + c]), ...);
+                    ((mine[Is] = Is == 0 ? T(0) : src[(size_t)D3Q19<Is>::opp * nc + c]), ...);
                 }(std::make_integer_sequence<int, 19>{});
                 auto bb = [&](auto Ic) {
                     constexpr int I = decltype(Ic)::value;
                     if constexpr (I > 0) {
                         const uint32_t t = sf[I] & 0x7fu;
-                        if (t == 1) f[I] = own[I];
-                        else if (t != 0) f[I] = Ar<T, E>::sub(own[I], T(p.lidc[D3Q19<I>::opp]));
+                        if (t == 1) f[I] = mine[I];
+                        else if (t != 0) f[I] = Ar<T, E>::sub(mine[I], T(p.lidc[D3Q19<I>::opp]));
                     }
                 };
                 [&]<int... Is>(std::integer_sequence<int, Is...>) { (bb(std::integral_constant<int, Is>{}), ...); }
                 (std::make_integer_sequence<int, 19>{});
             }
-#if ST_LBM_TMA_PROBE != 1
             if (MODE != LBM_STREAM) collide<T, E>(f, omega);
-#endif
         }
-#if ST_LBM_TMA_PROBE == 2
-        if (f[0] != T(-12345)) continue;
-#endif
         T* d = dst + c;
 #pragma unroll
         for (int i = 0; i < 19; ++i) d[(size_t)i * nc] = f[i];
-        }
     }
 }
 

@@ -2,6 +2,8 @@
 // SURVEY §8(f) f1): B = alpha*C + beta*F + gamma*E + delta*K over the 3x3x3
 // cube (centre, 6 faces, 12 edges, 8 corners), Jacobi two-grid sweeps,
 // Dirichlet shell (X1), dim_T levels kept on chip.
+// This kernel is the BIT-EXACT build (the oracle's X24 operation order); the
+// tolerance build runs st27t_kernel.cuh on the 7-point machinery.
 //
 // Mapping (B200, sm_100a).  One CTA = a 32 x 32 loaded XY tile (8 warps of
 // 32 lanes x 4 rows FP32, 32 x 16 with 2 rows FP64) streamed along a Z chunk,
@@ -107,25 +109,17 @@ __global__ void __launch_bounds__(NTHR, MINB) st27_kernel(const T* __restrict__ 
         st[j] = xin && yin;
     }
 
-    // FP32 tolerance build: rows travel as packed pairs (FADD2/FFMA2), pair k =
-    // rows (k, k + 2) of the thread's 4, so the y-neighbour pairs of one pair are
-    // the other pair (no pair construction but for the two edge rows)
-    constexpr bool PK = sizeof(T) == 4 && !EX && VY == 4;
     // Z windows: level L (0..D-1) as a source, slot k holds (a, f, e) of one plane
-    T wa[D][3][PK ? 1 : VY], wf[D][3][PK ? 1 : VY], we[D][3][PK ? 1 : VY];
-    float2 qa[D][3][PK ? 2 : 1], qf[D][3][PK ? 2 : 1], qe[D][3][PK ? 2 : 1];
+    T wa[D][3][VY], wf[D][3][VY], we[D][3][VY];
     // zero-initialised: the first rounds of a chunk read window slots that no
     // earlier round has written (their results are never stored, but reading
     // an indeterminate value is undefined behaviour the compiler may exploit)
 #pragma unroll
     for (int L = 0; L < D; ++L)
 #pragma unroll
-        for (int k = 0; k < 3; ++k) {
+        for (int k = 0; k < 3; ++k)
 #pragma unroll
-            for (int j = 0; j < (PK ? 1 : VY); ++j) wa[L][k][j] = wf[L][k][j] = we[L][k][j] = T(0);
-#pragma unroll
-            for (int j = 0; j < (PK ? 2 : 1); ++j) qa[L][k][j] = qf[L][k][j] = qe[L][k][j] = make_float2(0.f, 0.f);
-        }
+            for (int j = 0; j < VY; ++j) wa[L][k][j] = wf[L][k][j] = we[L][k][j] = T(0);
     // level-0 planes arrive PF-1 rounds ahead through a per-thread cp.async
     // ring (each thread copies and later reads only its own VY elements, so no
     // barrier guards the ring; the loads stay in flight across the rounds'
@@ -215,81 +209,6 @@ __global__ void __launch_bounds__(NTHR, MINB) st27_kernel(const T* __restrict__ 
             }
         }
     };
-    // packed FP32 round (tolerance build): same operations per point as round(),
-    // two rows per instruction; the level update contracts to FMUL2 + 3 FFMA2
-    const float2 al2 = make_float2((float)alpha, (float)alpha), be2 = make_float2((float)beta, (float)beta);
-    const float2 ga2 = make_float2((float)gamma, (float)gamma), de2 = make_float2((float)delta, (float)delta);
-    auto round_pk = [&](int i, auto Rc, auto Sc) {
-        constexpr int R = decltype(Rc)::value;
-        constexpr bool SHELL = decltype(Sc)::value;
-        constexpr int sN = (R + 2) % 3, sC = (R + 1) % 3, sM = R % 3;
-        float2 v[2];
-        issue(rslot == 0 ? PF - 1 : rslot - 1);
-        asm volatile("cp.async.wait_group %0;" ::"n"(PF - 1) : "memory");
-        {
-            const float* rr = reinterpret_cast<const float*>(&ring[rslot][w * VY][lane]);
-            v[0] = make_float2(rr[0], rr[2 * TW]);
-            v[1] = make_float2(rr[TW], rr[3 * TW]);
-        }
-        rslot = rslot == PF - 1 ? 0 : rslot + 1;
-#pragma unroll
-        for (int L = 0; L <= D; ++L) {
-            const int q = lo0 + i - L;
-            if (L > 0) {
-                const bool shz = q == 0 || q == p.nz - 1;
-#pragma unroll
-                for (int k = 0; k < 2; ++k) {
-                    const float2 c0 = qa[L - 1][sC][k];
-                    const float2 zs2 = __fadd2_rn(qa[L - 1][sM][k], qa[L - 1][sN][k]);
-                    const float2 F = __fadd2_rn(qf[L - 1][sC][k], zs2);
-                    const float2 E = __fadd2_rn(qe[L - 1][sC][k], __fadd2_rn(qf[L - 1][sM][k], qf[L - 1][sN][k]));
-                    const float2 K = __fadd2_rn(qe[L - 1][sM][k], qe[L - 1][sN][k]);
-                    const float2 r = __ffma2_rn(de2, K, __ffma2_rn(ga2, E, __ffma2_rn(be2, F, __fmul2_rn(al2, c0))));
-                    if constexpr (SHELL) {
-                        v[k].x = (shxy[k] || shz) ? c0.x : r.x;
-                        v[k].y = (shxy[k + 2] || shz) ? c0.y : r.y;
-                    } else {
-                        v[k] = r;
-                    }
-                }
-            }
-            if (L == D) {
-                if (q >= zs && q < ze) {
-                    float* ob = reinterpret_cast<float*>(b) + (size_t)q * plane;
-                    if (st[0]) ob[off32[0]] = v[0].x;
-                    if (st[1]) ob[off32[1]] = v[1].x;
-                    if (st[2]) ob[off32[2]] = v[0].y;
-                    if (st[3]) ob[off32[3]] = v[1].y;
-                }
-                break;
-            }
-            float* smf = reinterpret_cast<float*>(&sm[buf][0][0]);
-            smf[(w * VY) * TW + lane] = v[0].x;
-            smf[(w * VY + 3) * TW + lane] = v[1].y;
-            __syncthreads();
-            const float up = smf[max(w * VY - 1, 0) * TW + lane];
-            const float dn = smf[min(w * VY + VY, TH - 1) * TW + lane];
-            buf ^= 1;
-            // rows (0,2): y- = (up, v1), y+ = (v1, v3) = v[1]; rows (1,3): y- = v[0], y+ = (v2, dn)
-            const float2 vv0 = __fadd2_rn(make_float2(up, v[1].x), v[1]);
-            const float2 vv1 = __fadd2_rn(v[0], make_float2(v[0].y, dn));
-            const float2 vv[2] = {vv0, vv1};
-#pragma unroll
-            for (int k = 0; k < 2; ++k) {
-                const float2 xm = make_float2(__shfl_up_sync(0xffffffffu, v[k].x, 1), __shfl_up_sync(0xffffffffu, v[k].y, 1));
-                const float2 xp = make_float2(__shfl_down_sync(0xffffffffu, v[k].x, 1),
-                                              __shfl_down_sync(0xffffffffu, v[k].y, 1));
-                const float2 f = __fadd2_rn(__fadd2_rn(xm, xp), vv[k]);
-                const float2 vm = make_float2(__shfl_up_sync(0xffffffffu, vv[k].x, 1),
-                                              __shfl_up_sync(0xffffffffu, vv[k].y, 1));
-                const float2 vp = make_float2(__shfl_down_sync(0xffffffffu, vv[k].x, 1),
-                                              __shfl_down_sync(0xffffffffu, vv[k].y, 1));
-                qa[L][sN][k] = v[k];
-                qf[L][sN][k] = f;
-                qe[L][sN][k] = __fadd2_rn(vm, vp);
-            }
-        }
-    };
     // rotation chosen per round: the same three bodies called in sequence
     // from a loop stepping by three rounds gave wrong values from the fourth
     // round on (cause not isolated)
@@ -311,21 +230,6 @@ __global__ void __launch_bounds__(NTHR, MINB) st27_kernel(const T* __restrict__ 
         if (sh2) round(i + 2, std::integral_constant<int, 2>{}, S1{}); else round(i + 2, std::integral_constant<int, 2>{}, S0{});
     }
 #else
-    if constexpr (PK) {
-        for (int i = 0; i < nround; ++i) {
-            const int r = i % 3;
-            const bool sh = tile_shell || lo0 + i - D <= 0 || lo0 + i - 1 >= p.nz - 1;
-            if (sh) {
-                if (r == 0) round_pk(i, std::integral_constant<int, 0>{}, S1{});
-                else if (r == 1) round_pk(i, std::integral_constant<int, 1>{}, S1{});
-                else round_pk(i, std::integral_constant<int, 2>{}, S1{});
-            } else {
-                if (r == 0) round_pk(i, std::integral_constant<int, 0>{}, S0{});
-                else if (r == 1) round_pk(i, std::integral_constant<int, 1>{}, S0{});
-                else round_pk(i, std::integral_constant<int, 2>{}, S0{});
-            }
-        }
-    } else
     for (int i = 0; i < nround; ++i) {
         const int r = i % 3;
         const bool sh = tile_shell || lo0 + i - D <= 0 || lo0 + i - 1 >= p.nz - 1;
@@ -407,9 +311,10 @@ cudaError_t st27_launch(int dtype, bool exact, int D, const void* in, void* out,
     p.zchunk = 0;
     if (dtype == 0) { p.alpha = (float)alpha; p.beta = (float)beta; p.gamma = (float)gamma; p.delta = (float)delta; }
     else { p.alpha = alpha; p.beta = beta; p.gamma = gamma; p.delta = delta; }
-    if (dtype == 0)
-        return exact ? dispatch<float, true>(D, in, out, p, sms, s, grid_out) : dispatch<float, false>(D, in, out, p, sms, s, grid_out);
-    return exact ? dispatch<double, true>(D, in, out, p, sms, s, grid_out) : dispatch<double, false>(D, in, out, p, sms, s, grid_out);
+    // the tolerance build runs st27t_kernel.cuh (7-point machinery); this kernel is the bit-exact one
+    if (!exact) return cudaErrorInvalidValue;
+    return dtype == 0 ? dispatch<float, true>(D, in, out, p, sms, s, grid_out)
+                      : dispatch<double, true>(D, in, out, p, sms, s, grid_out);
 }
 
 }  // namespace st35d
