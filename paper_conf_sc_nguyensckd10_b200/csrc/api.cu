@@ -183,9 +183,10 @@ static St7LaunchFn lookup7(st_dtype dt, bool exact, int d, int vy, int nt, int m
 static int ctas_per_sm(const Geo7& g) { return g.minb == 9 ? 1 : g.minb; }
 
 static size_t smem7(const Geo7& g, st_dtype dt, int ring) {
-    // TMA ring + row exchange [D-1][2][2][threads] x 16 B + mbarriers + load cursor
-    return (size_t)ring * g.TX * g.TY * esize(dt) + (size_t)(g.d > 1 ? g.d - 1 : 0) * 4 * g.threads * 16 +
-           ST7_RING_MAX * 8;
+    // TMA ring + row exchange [D-1][2][2][threads] x one thread row (VX points: 16 B, or
+    // 8 B for the narrow FP32 layout) + mbarriers
+    return (size_t)ring * g.TX * g.TY * esize(dt) +
+           (size_t)(g.d > 1 ? g.d - 1 : 0) * 4 * g.threads * (g.VX * esize(dt)) + ST7_RING_MAX * 8;
 }
 
 // Planner for one sweep depth d over an nx x ny plane with nzo output planes:

@@ -22,7 +22,7 @@ cap lbm_tma_pull_256_f32 lbm_pull python tools/prof_lbm_k.py 256 6 f32 0
 cap lbm_tma_pull_1024_f32 lbm_pull python tools/prof_lbm_k.py 1024 4 f32 0
 cap lbm_push_256_f64 lbm_push python tools/prof_lbm_k.py 256 6 f64 0
 cap lbm_push_256_f32 lbm_push python tools/prof_lbm_k.py 256 6 f32 1
-cap st27_256_f32_d2 st27_kernel python tools/prof27.py 256 f32 2 12
+cap st27t_256_f32_d3 st27t python tools/prof27.py 256 f32 3 12
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:lbm_pull -s 2 -c 1 \
     -o $O/lbm_pull_full -f python tools/prof_lbm_k.py 256 6 f32 0 > $O/lbm_full.log 2>&1
 ncu -i $O/lbm_pull_full.ncu-rep --page raw --csv > $O/lbm_pull_full.raw.csv 2>/dev/null
