@@ -9,6 +9,7 @@
 #include <algorithm>
 #include <cudaTypedefs.h>
 #include <dlfcn.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include "../../include/st35d.h"
 #include "launch.h"
@@ -21,6 +22,15 @@ using namespace st35d;
 // NCCL CTAs per communicator (ncclConfig_t.maxCTAs): the ghost exchange is a few
 // MB per sweep, a handful of CTAs saturate NVLink for it, the rest stay with the sweep
 constexpr int ST_NCCL_MAX_CTAS = 4;
+
+// NVTX3 ranges (header-only; no cost without an attached tool): one per C-ABI
+// run and one per sweep / pass / ghost exchange, for nsys / ncu range filters
+struct NvtxRange {
+    explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange&) = delete;
+    NvtxRange& operator=(const NvtxRange&) = delete;
+};
 
 // ----------------------------------------------------------------------------
 // errors
@@ -624,6 +634,7 @@ static void split_work(int ntiles, int nzo, int d, int G, int* split, int zchunk
 }
 
 static int launch7(st_plan* p, const void* src, void* dst, int d, double alpha, double beta, const SlabView& sv) {
+    NvtxRange nvtx_("st7 sweep");
     Geo7* g = nullptr;
     int rc = get_geo7(p, d, sv.zb - sv.za, g);
     if (rc) return rc;
@@ -672,6 +683,7 @@ static int poll_nccl(st_plan* p) {
 }
 
 static int exchange_nccl(st_plan* p, void* buf, int d, int ncomp, cudaStream_t st) {
+    NvtxRange nvtx_("ghost exchange");
 #if ST_HAVE_NCCL
     Dist& D = p->dist;
     const size_t pb = (size_t)p->nx * p->ny * esize(p->dtype);
@@ -921,6 +933,7 @@ static int run7_device(st_plan* p, const void* in, void* out, double alpha, doub
 }
 
 extern "C" int st7_run(st_plan* p, const void* in, void* out, double alpha, double beta, int T) {
+    NvtxRange nvtx_("st7_run");
     if (!p) return fail(ST_EINVAL, "NULL plan");
     if (!in || !out) return fail(ST_EINVAL, "NULL grid pointer");
     if (T < 0) return fail(ST_EINVAL, "T = %d < 0", T);
@@ -949,6 +962,7 @@ extern "C" int st7_run(st_plan* p, const void* in, void* out, double alpha, doub
 // st27.cu kernel, D = min(dim_T, st27_depth_max()); single process only.
 // ----------------------------------------------------------------------------
 static int launch27t(st_plan* p, const void* src, void* dst, int d, const double w[4]) {
+    NvtxRange nvtx_("st27 sweep");
     Geo7 g;
     int rc = plan27t(p, d, p->nz, g);
     if (rc) return rc;
@@ -1004,6 +1018,7 @@ static int run27_device(st_plan* p, const void* in, void* out, const double w[4]
 
 extern "C" int st27_run(st_plan* p, const void* in, void* out, double alpha, double beta, double gamma, double delta,
                         int T) {
+    NvtxRange nvtx_("st27_run");
     if (!p) return fail(ST_EINVAL, "NULL plan");
     if (!in || !out) return fail(ST_EINVAL, "NULL grid pointer");
     if (T < 0) return fail(ST_EINVAL, "T = %d < 0", T);
@@ -1034,6 +1049,7 @@ extern "C" int st27_run(st_plan* p, const void* in, void* out, double alpha, dou
 // process only.
 // ----------------------------------------------------------------------------
 static int launch13(st_plan* p, const void* src, void* dst, int d, const double w[3]) {
+    NvtxRange nvtx_("st13 sweep");
     Geo7 g;
     int rc = plan13(p, d, p->nz, g);
     if (rc) return rc;
@@ -1080,6 +1096,7 @@ static int run13_device(st_plan* p, const void* in, void* out, const double w[3]
 }
 
 extern "C" int st13_run(st_plan* p, const void* in, void* out, double alpha, double beta, double gamma, int T) {
+    NvtxRange nvtx_("st13_run");
     if (!p) return fail(ST_EINVAL, "NULL plan");
     if (!in || !out) return fail(ST_EINVAL, "NULL grid pointer");
     if (T < 0) return fail(ST_EINVAL, "T = %d < 0", T);
@@ -1298,6 +1315,7 @@ static bool lbm_use_push(const st_plan* p) {
 }
 
 static int launch_lbm35(st_plan* p, const void* src, void* dst, int d, double omega, const SlabView& sv) {
+    NvtxRange nvtx_("lbm 3.5D sweep");
     GeoL g;
     int rc = planL(p, d, g);
     if (rc) return rc;
@@ -1322,6 +1340,7 @@ static int launch_lbm35(st_plan* p, const void* src, void* dst, int d, double om
 
 static int launch_lbm(st_plan* p, const void* src, void* dst, const uint8_t* flags, double omega,
                       const SlabView& sv) {
+    NvtxRange nvtx_("lbm push step");
     LbmParams prm{};
     prm.nx = p->nx; prm.ny = p->ny; prm.nzb = sv.nzb; prm.zbase = sv.zbase; prm.nzg = p->nz;
     prm.za = sv.za; prm.zb = sv.zb;
@@ -1427,6 +1446,7 @@ static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T
         void* a = fsrc;
         void* b = fdst;
         auto pass = [&](int mode, void* from, void* to) -> int {
+            NvtxRange nvtx_(mode == LBM_COLLIDE ? "lbm collide pass" : mode == LBM_PULL ? "lbm pull pass" : "lbm stream pass");
             cudaError_t e;
             if (tma)
                 e = lbm_pull_tma_launch(dt, p->exact, mode, p->opt_pdl != 0, from == fsrc ? map_src : map_dst, from,
@@ -1457,6 +1477,7 @@ static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T
 }
 
 extern "C" int lbm_d3q19_run(st_plan* p, void* fsrc, void* fdst, double omega, int T, const uint8_t* flags) {
+    NvtxRange nvtx_("lbm_d3q19_run");
     if (!p) return fail(ST_EINVAL, "NULL plan");
     if (!fsrc || !fdst || !flags) return fail(ST_EINVAL, "NULL pointer");
     if (T < 0) return fail(ST_EINVAL, "T = %d < 0", T);
