@@ -378,3 +378,24 @@ def test_gather_form_tma_pulls_256(oracle_lib, dtype):
             assert np.array_equal(got, ref)
         else:
             assert relerr(got, ref) <= TOL[dtype]
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_host_pointers(oracle_lib, dtype):
+    # host (numpy) lattices and flags: staged through plan-owned device buffers, the call
+    # synchronises; T = 5 takes the TMA gather form for FP32 and the push kernel for FP64
+    nx, ny, nz = 64, 20, 11
+    flags = stgen.cavity_flags(nx, ny, nz)
+    flags[5, 8:10, 20:23] = stgen.WALL
+    f0 = stgen.lbm_random(nx, ny, nz, 37, dtype)
+    ref = oracle_lib.lbm(f0, flags, 1.6, 5)
+    for exact in (True, False):
+        with st.Plan(nx, ny, nz, torch.float32 if dtype == np.float32 else torch.float64, 1) as p:
+            p.set_bitexact(exact)
+            out = np.empty_like(f0)
+            p.lbm(f0.copy(), out, 1.6, 5, flags.copy())
+            assert p.info(True)["kernel"] == (400 if dtype == np.float32 else 100)
+        if exact:
+            assert np.array_equal(out, ref)
+        else:
+            assert relerr(out, ref) <= TOL[dtype]
