@@ -499,7 +499,9 @@ def main():
                                             "ms_per_step": round(msl, 3),
                                             "roofline": {"bound": "hbm", "achieved": round(gbs, 1),
                                                          "peak": hbm_gbs, "unit": "GB/s",
-                                                         "frac": round(gbs / hbm_gbs, 4)},
+                                                         "frac": round(gbs / hbm_gbs, 4),
+                                                         "traffic": load_traffic(f"lbm_{dtn}_256_D1"),
+                                                         "algorithmic_bytes_per_pass": LBM_BYTES[E] * nl ** 3},
                                             "launches": pl.last_launches(),
                                             "kernel": pl.info(True)["kernel"]}
             del fa, fb, f0, flags
@@ -533,7 +535,9 @@ def main():
                                           "kernel": pl.info(True)["kernel"],
                                           "note": "configs[4] lattice on one GPU (strong-scaling base)",
                                           "roofline": {"bound": "hbm", "achieved": round(gbs, 1), "peak": hbm_gbs,
-                                                       "unit": "GB/s", "frac": round(gbs / hbm_gbs, 4)}}
+                                                       "unit": "GB/s", "frac": round(gbs / hbm_gbs, 4),
+                                                       "traffic": load_traffic("lbm_f32_1024_D1"),
+                                                       "algorithmic_bytes_per_pass": LBM_BYTES[4] * nb ** 3}}
             del fa, fb, flb
             torch.cuda.empty_cache()
     cpu = cpu_baseline_7pt(n, T) if (rank == 0 and world == 1) else None
