@@ -204,9 +204,10 @@ lbm_pull_tma_kernel(const __grid_constant__ CUtensorMap mapn, const __grid_const
     }
 }
 
-// tile width for a lattice row of nx cells (measured on B200, FP32 cavity, GLUPS:
-// 256^3 64 x 4 34.1 vs 128 x 2 30.8; 1024^3 64 x 4 25.0 vs 128 x 2 30.0)
-static int pull_bx(int dtype, int nx) { return dtype == 0 ? (nx >= 512 ? 128 : 64) : 32; }
+// tile width for a lattice row of nx cells (measured on B200, FP32 cavity, GLUPS,
+// 64 x 4 vs 128 x 2 tiles: 256^3 34.1 / 30.8, 384^3 31.6 / 31.5, 512^3 35.0 / 32.9,
+// 640^3 31.2 / 33.4, 1024^3 25.0 / 30.6)
+static int pull_bx(int dtype, int nx) { return dtype == 0 ? (nx > 512 ? 128 : 64) : 32; }
 
 template <typename T, int BX>
 static size_t stage_bytes() { return 19u * PullTile<T, BX>::SLOT * sizeof(T); }
