@@ -167,15 +167,15 @@ int st_plan_set_variant(st_plan* plan, int variant);
  *                       batched-flag push kernel; 0 / 1 force the per-direction /
  *                       batched kernel (FP64 always batches).
  *   ST_OPT_LBM_KERNEL   0 (default) auto: when the plan's LBM depth is 1, the
- *                       TMA gather form (4) for FP32 single-domain runs of T >= 4
- *                       with nx * 4 % 16 == 0, else the dim_T = 1 push kernel; at
- *                       depth >= 2 the multi-level on-chip kernel; 1 push
- *                       (dim_T = 1 sweeps); 2 multi-level kernel at the plan depth;
- *                       3 gather form (collide pass, T-1 pull passes, stream pass;
- *                       aligned stores; single domain); 4 the same with the
- *                       pull passes fed by TMA (4D boxes shifted per population,
- *                       S-stage shared-memory ring; needs nx * sizeof(T) % 16 == 0,
- *                       else the plain pull kernel runs).
+ *                       TMA gather form (4) for FP32 runs of T >= 4, else the
+ *                       dim_T = 1 push kernel; at depth >= 2 the multi-level
+ *                       on-chip kernel; 1 push (dim_T = 1 sweeps); 2 multi-level
+ *                       kernel at the plan depth; 3 gather form (collide pass,
+ *                       T-1 pull passes, stream pass; aligned stores; single
+ *                       domain); 4 the same with every pass fed by TMA (boxes
+ *                       shifted per population, S-stage shared-memory ring); on
+ *                       Z slabs the T + 1 passes run as depth-1 sweeps of the
+ *                       slab schedule (one ghost plane per face per pass).
  *   ST_OPT_LBM_STAGES   0 (default) auto; 1..8 stages of the TMA pull ring.
  *   ST_OPT_OVERLAP      1 (default): Z-slab ghost exchange overlapped with the
  *                       interior sweep on a side stream; 0 serialised.

@@ -810,7 +810,7 @@ static int run_sweeps(st_plan* p, const std::vector<int>& ds, const void* in, vo
         for (size_t k = 0; k < ds.size(); ++k) {
             SlabView sv;
             sv.stream = p->stream; sv.flags = flags; sv.fl2 = p->fl2;
-            sv.nzb = p->nz; sv.zbase = 0; sv.za = 0; sv.zb = p->nz; sv.single = true;
+            sv.nzb = p->nz; sv.zbase = 0; sv.za = 0; sv.zb = p->nz; sv.single = true; sv.sweep = (int)k;
             int rc = launch(src, dst, ds[k], sv);
             if (rc) return rc;
             src = bufs[(k + 1) % 2];
@@ -842,8 +842,9 @@ static int run_sweeps(st_plan* p, const std::vector<int>& ds, const void* in, vo
         if (loop) return exchange_loop(p, which, d, ncomp, st);
         return exchange_nccl(p, sl[0].buf[which], d, ncomp, st);
     };
-    auto view = [&](const S& s, int za, int zb, int cap) {
+    auto view = [&](const S& s, int za, int zb, int cap, int sweep) {
         SlabView sv;
+        sv.sweep = sweep;
         sv.nzb = s.nzb; sv.zbase = s.z0 - D.g; sv.za = za; sv.zb = zb;
         sv.flags = s.flags; sv.fl2 = s.fl2; sv.single = false; sv.stream = p->stream; sv.grid_cap = cap;
         return sv;
@@ -875,7 +876,7 @@ static int run_sweeps(st_plan* p, const std::vector<int>& ds, const void* in, vo
                 for (size_t k = 0; k < sl.size(); ++k) {
                     const SlabStep& stp = sched[k][i];
                     rc = launch(sl[k].buf[stp.src], sl[k].buf[1 - stp.src], stp.depth,
-                                view(sl[k], stp.z_begin, stp.z_end, stp.grid_cap ? cap : 0));
+                                view(sl[k], stp.z_begin, stp.z_end, stp.grid_cap ? cap : 0, stp.sweep));
                     if (rc) return rc;
                 }
                 cur = 1 - st0.src;
@@ -1362,6 +1363,43 @@ static int launch_lbm(st_plan* p, const void* src, void* dst, const uint8_t* fla
     return ST_OK;
 }
 
+// one pass of the TMA gather form over the output planes [sv.za, sv.zb) of a
+// (slab) buffer of sv.nzb planes (Z-slab schedule; the single-domain path
+// encodes its maps once per run instead)
+static int launch_lbm_tma_slab(st_plan* p, int mode, const void* src, void* dst, double omega, const SlabView& sv) {
+    NvtxRange nvtx_(mode == LBM_COLLIDE ? "lbm collide pass" : mode == LBM_PULL ? "lbm pull pass" : "lbm stream pass");
+    if (sv.zb <= sv.za) return ST_OK;
+    const int dt = p->dtype == ST_F32 ? 0 : 1;
+    int bx, by, halo;
+    lbm_pull_tma_box(dt, p->nx, &bx, &by, &halo);
+    CUtensorMap maps[2];
+    for (int w = 0; w < 2; ++w) {
+        int rc = encode_lbm(&maps[w], src, p->dtype, p->nx, p->ny, sv.nzb, bx + w * halo, by);
+        if (rc) return rc;
+    }
+    LbmParams prm{};
+    prm.nx = p->nx; prm.ny = p->ny; prm.nzb = sv.nzb; prm.zbase = sv.zbase; prm.nzg = p->nz;
+    prm.za = sv.za; prm.zb = sv.zb;
+    prm.omega = omega;
+    if (p->dtype == ST_F32) lid_coeffs<float>(p->lid, prm.lidc);
+    else lid_coeffs<double>(p->lid, prm.lidc);
+    const size_t sb = lbm_pull_tma_stage_bytes(dt, p->nx);
+    const int stages = p->opt_lbm_stages > 0 ? p->opt_lbm_stages : (dt == 0 ? 3 : 1);
+    if ((size_t)stages * sb > p->smem_optin) return fail(ST_EUNSUPPORTED, "LBM pull ring of %d stages", stages);
+    const int per_sm = std::max(1, std::min(2, (int)(p->smem_sm / ((size_t)stages * sb + 1024))));
+    const int tcols = (p->nx + bx - 1) / bx;
+    const long long tiles = (long long)tcols * ((p->ny + by - 1) / by) * (sv.zb - sv.za);
+    long long cap = (long long)p->sms * per_sm;
+    if (sv.grid_cap > 0) cap = std::min<long long>(cap, (long long)sv.grid_cap * per_sm);   // SMs left to NCCL
+    int grid = (int)std::min<long long>(tiles, cap);
+    if (grid > 1 && grid % tcols == 0) --grid;   // rotate the x-wall tiles over the CTAs (see runlbm_device)
+    cudaError_t e = lbm_pull_tma_launch(dt, p->exact, mode, p->opt_pdl != 0, maps, src, dst, sv.fl2, prm, grid,
+                                        stages, sv.stream ? sv.stream : p->stream);
+    if (e != cudaSuccess) return fail(ST_ECUDA, "lbm TMA pass: %s", cudaGetErrorString(e));
+    ++p->launches;
+    return ST_OK;
+}
+
 static int check_shell(st_plan* p, const uint8_t* flags) {
     if (p->flags_checked == flags) return ST_OK;
     if (p->dist.mode == Dist::NCCL) { p->flags_checked = flags; return ST_OK; }  // caller-owned slab flags
@@ -1399,15 +1437,27 @@ static int runlbm_device(st_plan* p, void* fsrc, void* fdst, double omega, int T
         cudaError_t e = lbm_fl2(flags, p->fl2, p->nx, p->ny, p->dist.nzb, p->stream);
         if (e != cudaSuccess) return fail(ST_ECUDA, "fl2 prepass: %s", cudaGetErrorString(e));
     }
-    // FP32 single-domain dim_T = 1 runs of T >= 4 steps: the gather form with TMA-fed
-    // pull passes (measured on B200, 256^3 cavity: 33.1 vs 25.8 GLUPS for the push
-    // kernel; FP64 keeps push, 18.4 vs 16.7).  T + 1 passes.
+    // FP32 dim_T = 1 runs of T >= 4 steps: the gather form with TMA-fed passes
+    // (measured on B200, 256^3 cavity: 34.1 vs 25.8 GLUPS for the push kernel; FP64
+    // keeps push, 18.4 vs 16.7).  T + 1 passes.
+    // Z slabs run the same T + 1 passes as depth-1 sweeps of the slab schedule
+    // (one ghost plane per face exchanged before each pull / stream pass).
     int gk = p->opt_lbm_kernel;
-    if (gk == 0 && push && p->dist.mode == Dist::SINGLE && p->dtype == ST_F32 && T >= 4 &&
-        ((size_t)p->nx * esize(p->dtype)) % 16 == 0)
+    if (gk == 0 && push && p->dtype == ST_F32 && T >= 4 && ((size_t)p->nx * esize(p->dtype)) % 16 == 0)
         gk = 4;
+    if (gk == 4 && p->dist.mode != Dist::SINGLE) {
+        p->last_lbm_kernel = 400;
+        rc = run_sweeps(p, std::vector<int>(T + 1, 1), fsrc, fdst, 19, flags,
+                        [&](const void* a, void* b, int, const SlabView& sv) {
+                            const int mode = sv.sweep == 0 ? LBM_COLLIDE : (sv.sweep == T ? LBM_STREAM : LBM_PULL);
+                            return launch_lbm_tma_slab(p, mode, a, b, omega, sv);
+                        });
+        if (rc) return rc;
+        CUDA_TRY(cudaGetLastError());
+        return ST_OK;
+    }
     if (gk == 3 || gk == 4) {   // gather form: C, T-1 pulls, S (single domain)
-        if (p->dist.mode != Dist::SINGLE) return fail(ST_EUNSUPPORTED, "the gather-form LBM kernels are single-domain");
+        if (p->dist.mode != Dist::SINGLE) return fail(ST_EUNSUPPORTED, "the plain gather-form LBM kernels are single-domain");
         LbmParams prm{};
         prm.nx = p->nx; prm.ny = p->ny; prm.nzb = p->nz; prm.zbase = 0; prm.nzg = p->nz;
         prm.za = 0; prm.zb = p->nz;

@@ -31,6 +31,7 @@ struct SlabView {
     uint8_t* fl2 = nullptr;           // LBM neighbour-flag buffer of this slab (nzb planes)
     bool single = true;           // the whole grid in one buffer
     int grid_cap = 0;             // >0: leave SMs free (overlapped NCCL kernels)
+    int sweep = 0;                // index of the sweep (pass) this launch belongs to
     cudaStream_t stream = nullptr;
 };
 

@@ -79,18 +79,21 @@ lbm_pull_tma_kernel(const __grid_constant__ CUtensorMap mapn, const __grid_const
     pdl_trigger();
     pdl_wait();   // the previous pass's writes are visible from here on
 
-    const int nx = p.nx, ny = p.ny, nz = p.nzb;
+    // buffer planes [za, zb) (Z slabs: the owned planes or a part of them; the
+    // buffer holds nz = nzb planes, global plane = zbase + buffer plane)
+    const int nx = p.nx, ny = p.ny, nz = p.nzb, za = p.za;
+    const int zs0 = -p.zbase, zs1 = p.nzg - 1 - p.zbase;   // buffer planes of the global z shell
     // tiles dealt round-robin (x fastest): at any moment the CTAs stream
     // neighbouring tiles of the same planes, so each population's rows are read
     // in address order across the chip and a tile's x halo is its neighbour's
     // edge, fetched by the next CTA at the same time (measured: contiguous tile
     // ranges per CTA scatter the reads over the lattice, 17 vs 26 GLUPS)
-    const long long ntiles = (long long)tiles_x * tiles_y * nz;
+    const long long ntiles = (long long)tiles_x * tiles_y * (p.zb - p.za);
     const long long t_begin = blockIdx.x, t_end = ntiles, t_step = gridDim.x;
     auto where = [&](long long tile, int& x0, int& y0, int& z) {
         const int tx = (int)(tile % tiles_x);
         const long long r = tile / tiles_x;
-        x0 = tx * BX; y0 = (int)(r % tiles_y) * BY; z = (int)(r / tiles_y);
+        x0 = tx * BX; y0 = (int)(r % tiles_y) * BY; z = za + (int)(r / tiles_y);
     };
     if (tid >= NC) {   // producer warp: one lane issues the TMA loads
         if (tid == NC) {
@@ -103,7 +106,7 @@ lbm_pull_tma_kernel(const __grid_constant__ CUtensorMap mapn, const __grid_const
                 int x0, y0, z;
                 where(tile, x0, y0, z);
                 // shell planes (copied through) and the collide pass: own (unshifted) values
-                const bool own = MODE == LBM_COLLIDE || z == 0 || z == nz - 1;
+                const bool own = MODE == LBM_COLLIDE || z == zs0 || z == zs1;
                 T* b = buf + (size_t)s * 19 * SLOT;
                 if (own) {
                     mbar_arrive_expect_tx(&full[s], TX_SHELL);
@@ -142,7 +145,7 @@ lbm_pull_tma_kernel(const __grid_constant__ CUtensorMap mapn, const __grid_const
         where(tile, x0, y0, z);
         const uint32_t fl = fl_next;
         if (tile + t_step < t_end) fl_next = flag_of(tile + t_step);
-        const bool own = MODE == LBM_COLLIDE || z == 0 || z == nz - 1;   // unshifted boxes
+        const bool own = MODE == LBM_COLLIDE || z == zs0 || z == zs1;   // unshifted boxes
         const int x = x0 + cx, y = y0 + cy;
         const bool inb = x < nx && y < ny;
         const size_t c = (size_t)z * plane + (size_t)y * nx + x;

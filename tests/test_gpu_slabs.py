@@ -120,3 +120,33 @@ def test_nccl_one_rank_communicator(oracle_lib, kind, overlap):
             p.sync()
             got = y.cpu().numpy()[:, g:g + nz]
         assert np.array_equal(got, oracle_lib.lbm(f0, flags, 1.6, T))
+
+
+@pytest.mark.parametrize("P", [2, 3, 4])
+@pytest.mark.parametrize("T", [4, 7])
+def test_lbm_loopback_tma_gather(oracle_lib, P, T):
+    # FP32 dim_T = 1 runs of T >= 4 take the TMA gather form on Z slabs too: T + 1
+    # passes as depth-1 sweeps of the slab schedule (one ghost plane exchanged per
+    # face before each pull / stream pass, boundary planes first, interior overlapped);
+    # bit-identical to the oracle in the exact build, within the gate otherwise
+    nx, ny, nz = 64, 20, 26
+    flags = stgen.cavity_flags(nx, ny, nz)
+    flags[12:15, 5:9, 20:30] = stgen.WALL    # obstacle across a slab boundary
+    flags[7, 10, 40] = stgen.LID
+    f0 = stgen.lbm_random(nx, ny, nz, 41, np.float32)
+    ref = oracle_lib.lbm(f0, flags, 1.6, T)
+    for exact in (True, False):
+        with st.Plan(nx, ny, nz, torch.float32, 1) as p:
+            p.set_bitexact(exact)
+            st.st_plan_set_loopback_slabs(p.h, P)
+            a = torch.from_numpy(f0).cuda()
+            b = torch.empty_like(a)
+            p.lbm(a, b, 1.6, T, torch.from_numpy(flags).cuda())
+            p.sync()
+            assert p.info(True)["kernel"] == 400
+            got = b.cpu().numpy()
+        if exact:
+            assert np.array_equal(got, ref), (P, T)
+        else:
+            g = got.astype(np.float64)
+            assert float(np.max(np.abs(g - ref) / np.maximum(np.abs(ref), 1e-30))) <= 1e-4
